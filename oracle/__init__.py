@@ -60,7 +60,7 @@ def _get():
         L.oracle_fit.restype = d
         L.oracle_fit.argtypes = [i32, i32, d, i64, p, p, p, p]
         L.oracle_factorize.argtypes = [i32, p, i64, p, p, d, i32, i32, d, d, i32, d, i32, i32, i32,
-                                       p, p, p, p, p, p]
+                                       p, p, p, p, p, p, p]
         _lib = L
     return _lib
 
@@ -218,7 +218,8 @@ def factorize(X: Tensor, factors, outer_iters=10, tol=1e-2, max_iter=10, rho=0.0
               warm=WARM_SCALED, normalize_init=True, prox=PROX_NONNEG, fit_tol=0.0):
     """O9/O11: Alg. 1 (L476-506) with readings D4, D6, D11, D13.
 
-    Returns dict(factors, lam (N x R), fit[outer_done], iters[outer_done x N], phase_ms[4])."""
+    Returns dict(factors, lam (N x R), fit[outer_done], iters[outer_done x N], phase_ms[4],
+    trace[outer_done x N x max_iter x 4] of the ADMM sums)."""
     N = X.nmodes
     R = factors[0].shape[1]
     H = [np.array(f, dtype=np.float64, copy=True, order="C") for f in factors]
@@ -227,13 +228,16 @@ def factorize(X: Tensor, factors, outer_iters=10, tol=1e-2, max_iter=10, rho=0.0
     iters = np.zeros((outer_iters, N), dtype=np.int32)
     done = ctypes.c_int()
     phase = np.zeros(4)
+    trace = np.zeros((outer_iters, N, max_iter, 4))
     dims_a = np.asarray(X.dims, dtype=np.int64)
     st = _get().oracle_factorize(N, dims_a.ctypes.data, X.nnz, _ptrs(X.idx), X.vals.ctypes.data,
                                  float(X.normX2), R, int(outer_iters), float(fit_tol), float(tol),
                                  int(max_iter), float(rho), int(warm), int(bool(normalize_init)),
                                  int(prox), _ptrs(H), lam.ctypes.data, fits.ctypes.data,
-                                 iters.ctypes.data, ctypes.byref(done), phase.ctypes.data)
+                                 iters.ctypes.data, ctypes.byref(done), phase.ctypes.data,
+                                 trace.ctypes.data)
     if st:
         raise OracleError(st, "factorize")
     d = done.value
-    return dict(factors=H, lam=lam, fit=fits[:d], iters=iters[:d], phase_ms=phase)
+    return dict(factors=H, lam=lam, fit=fits[:d], iters=iters[:d], phase_ms=phase, trace=trace[:d],
+                tol=tol)

@@ -411,12 +411,14 @@ double oracle_fit(int N, int R, double normX2, int64_t I_last, const double* M_l
  *   ADMM(S, M, H, U^(n)); (H^(n), lambda^(n)) = normalize(H); G^(n) = H^(n)T H^(n)
  * then fit; stop early if fit_tol > 0 and |fit - fit_prev| < fit_tol (D11).
  * lam_all: N*R output (every mode's lambda; the Kruskal lambda is the last mode's, D10).
- * phase_ms[4] += GRAM, MTTKRP, UPDATE, NORMALIZE wall times. */
+ * phase_ms[4] += GRAM, MTTKRP, UPDATE, NORMALIZE wall times.
+ * trace_out (optional) [outer_iters][N][max_iter][4]: the four sums of every ADMM
+ * pass (r, s, nH, nU), used by tests to measure the stop-test margin (U2). */
 int oracle_factorize(int N, const int64_t* dims, int64_t nnz, const int32_t* const* cidx,
                      const double* cvals, double normX2, int R, int outer_iters, double fit_tol,
                      double tol, int max_iter, double rho_in, int warm, int normalize_init, int prox,
                      double* const* H, double* lam_all, double* fit_out, int* iters_out,
-                     int* outer_done, double* phase_ms) {
+                     int* outer_done, double* phase_ms, double* trace_out) {
   if (N < 2 || N > 8 || R < 1 || R > 128 || outer_iters < 1 || max_iter < 1) return ORC_EINVAL;
   int st = ORC_OK;
   double* G[8]; double* U[8];
@@ -452,7 +454,8 @@ int oracle_factorize(int N, const int64_t* dims, int64_t nnz, const int32_t* con
           for (int c = 0; c < R; c++) H[n][i * R + c] = H[n][i * R + c] * lam[c];
       }
       double stats[6];
-      st = oracle_admm(dims[n], R, M, S, H[n], U[n], tol, max_iter, rho_in, prox, stats, NULL);
+      double* tr = trace_out ? trace_out + ((size_t)t * N + n) * (size_t)max_iter * 4 : NULL;
+      st = oracle_admm(dims[n], R, M, S, H[n], U[n], tol, max_iter, rho_in, prox, stats, tr);
       if (st) break;
       if (iters_out) iters_out[t * N + n] = (int)stats[0];
       double t3 = now_ms();

@@ -1,0 +1,321 @@
+// extern "C" entry points of libcstf (include/cstf.h) and the Alg. 1 driver.
+#include <cstring>
+#include <vector>
+
+#include "internal.h"
+
+using namespace cstf;
+
+namespace {
+
+cudaStream_t S(void* s) { return static_cast<cudaStream_t>(s); }
+
+bool rank_ok(int R) { return R >= 1 && R <= 128; }
+
+// Device-side scratch of one factorize / admm_update call, cached per device.
+struct DriverWs {
+  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac;
+  double* host_small = nullptr;  // pinned: fit, flags
+};
+DriverWs& dws() {
+  static thread_local DriverWs w[64];
+  int dev = 0;
+  cudaGetDevice(&dev);
+  DriverWs& r = w[dev & 63];
+  if (!r.host_small) cudaMallocHost(&r.host_small, 64 * sizeof(double));
+  return r;
+}
+
+cstf_status check_flag(const int* d_flag, cudaStream_t st) {
+  int f = 0;
+  CSTF_CUDA(cudaMemcpyAsync(&f, d_flag, 4, cudaMemcpyDeviceToHost, st));
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  if (f & 1) return fail(CSTF_ERR_NOT_SPD, "S + rho I is not positive definite (rho <= 0 or pivot <= 0)");
+  if (f & 2) return fail(CSTF_ERR_NUMERIC, "non-finite ADMM residual or fit");
+  return CSTF_OK;
+}
+
+struct PhaseTimer {
+  bool on = false;
+  cudaStream_t st = nullptr;
+  std::vector<cudaEvent_t> ev;
+  std::vector<int> mode, phase;   // segment k: ev[2k] .. ev[2k+1]
+  std::vector<int64_t> l0;
+  double* phase_ms = nullptr;
+  double* mode_phase_ms = nullptr;
+  int64_t* mode_launches = nullptr;
+  int nseg = 0;
+  int64_t launch_mark = 0;
+  ~PhaseTimer() { for (auto e : ev) cudaEventDestroy(e); }
+  void begin(int m, int p) {
+    launch_mark = cstf_kernel_launch_count();
+    if (!on) return;
+    if ((size_t)(2 * nseg + 2) > ev.size()) {
+      for (int k = 0; k < 2; k++) { cudaEvent_t e; cudaEventCreate(&e); ev.push_back(e); }
+    }
+    cudaEventRecord(ev[2 * nseg], st);
+    if ((size_t)nseg >= mode.size()) { mode.push_back(m); phase.push_back(p); }
+    else { mode[nseg] = m; phase[nseg] = p; }
+  }
+  void end(int m, int p) {
+    if (mode_launches) mode_launches[m * CSTF_NUM_PHASES + p] += cstf_kernel_launch_count() - launch_mark;
+    if (!on) return;
+    cudaEventRecord(ev[2 * nseg + 1], st);
+    nseg++;
+  }
+  // after a stream sync: accumulate and reset
+  void collect() {
+    for (int k = 0; k < nseg; k++) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, ev[2 * k], ev[2 * k + 1]);
+      if (phase_ms) phase_ms[phase[k]] += ms;
+      if (mode_phase_ms) mode_phase_ms[mode[k] * CSTF_NUM_PHASES + phase[k]] += ms;
+    }
+    nseg = 0;
+  }
+};
+
+cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_comm* comm,
+                           double* const* d_factors, double* d_lambda, cstf_report* rep,
+                           cudaStream_t st) {
+  const int N = X->N;
+  const int R = o->R;
+  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
+  if (comm_nranks(comm) > 1) return fail(CSTF_ERR_UNSUPPORTED, "distributed factorize: use a partitioned tensor");
+  for (int n = 0; n < N; n++)
+    if (!d_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");
+  DriverWs& w = dws();
+  int64_t Imax = 0, Usum = 0;
+  for (int n = 0; n < N; n++) { Imax = std::max(Imax, X->dims[n]); Usum += X->dims[n] * R; }
+  CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
+  CSTF_TRY(w.lam.ensure((size_t)N * R * 8));
+  CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
+  CSTF_TRY(w.scal.ensure(64));
+  CSTF_TRY(w.flag.ensure(64));
+  CSTF_TRY(w.fitbuf.ensure(300 * 8));
+  CSTF_TRY(w.M.ensure((size_t)Imax * R * 8));
+  CSTF_TRY(w.U.ensure((size_t)Usum * 8));
+  double* G = w.grams.as<double>();
+  double* lam = w.lam.as<double>();
+  double* M = w.M.as<double>();
+  int* flag = w.flag.as<int>();
+  std::vector<double*> U(N);
+  {
+    int64_t off = 0;
+    for (int n = 0; n < N; n++) { U[n] = w.U.as<double>() + off; off += X->dims[n] * R; }
+  }
+  CSTF_CUDA(cudaMemsetAsync(flag, 0, 4, st));
+  CSTF_CUDA(cudaMemsetAsync(w.U.p, 0, (size_t)Usum * 8, st));
+  // init (Alg. 1 l.1-5; readings D6): normalise, lambda = 1, G = H^T H
+  for (int n = 0; n < N; n++) {
+    double* Gn = G + (size_t)n * R * R;
+    CSTF_TRY(gram_raw(d_factors[n], X->dims[n], R, Gn, st));
+    if (o->normalize_init) CSTF_TRY(normalize_from_gram(d_factors[n], X->dims[n], R, Gn, lam + n * R, st));
+    CSTF_TRY(fill(lam + n * R, R, 1.0, st));
+  }
+  PhaseTimer tm;
+  tm.on = o->timing != 0;
+  tm.st = st;
+  if (rep) {
+    tm.phase_ms = rep->phase_ms;
+    tm.mode_phase_ms = rep->mode_phase_ms;
+    tm.mode_launches = rep->mode_launches;
+    if (rep->phase_ms) for (int p = 0; p < CSTF_NUM_PHASES; p++) rep->phase_ms[p] = 0.0;
+    if (rep->mode_phase_ms) for (int p = 0; p < N * CSTF_NUM_PHASES; p++) rep->mode_phase_ms[p] = 0.0;
+    if (rep->mode_launches) for (int p = 0; p < N * CSTF_NUM_PHASES; p++) rep->mode_launches[p] = 0;
+    rep->outer_done = 0;
+  }
+  double fit_prev = 0.0;
+  for (int t = 0; t < o->outer_iters; t++) {
+    for (int n = 0; n < N; n++) {
+      const int64_t I = X->dims[n];
+      double* Gn = G + (size_t)n * R * R;
+      // a1 + a3 + a4: S = *_{k!=n} G^(k), rho, Cholesky, Inv   (GRAM phase)
+      tm.begin(n, CSTF_PHASE_GRAM);
+      CSTF_TRY(chol_inverse(nullptr, G, N, n, R, o->admm.rho, w.inv.as<double>(), w.scal.as<double>(), flag, st));
+      tm.end(n, CSTF_PHASE_GRAM);
+      // a2: MTTKRP
+      tm.begin(n, CSTF_PHASE_MTTKRP);
+      CSTF_TRY(mttkrp(X, n, R, d_factors, M, st, nullptr));
+      tm.end(n, CSTF_PHASE_MTTKRP);
+      // a5: ADMM, warm start H^(n) diag(lambda^(n)) (D4) unless the literal reading
+      tm.begin(n, CSTF_PHASE_UPDATE);
+      AdmmArgs a;
+      a.M = M; a.H = d_factors[n]; a.U = U[n];
+      a.hscale = (o->warm == CSTF_WARM_SCALED) ? lam + n * R : nullptr;
+      a.I = I; a.R = R; a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
+      a.tol = o->admm.tol; a.max_iter = o->admm.max_iter; a.prox = o->admm.prox; a.variant = o->admm.variant;
+      int iters = 0;
+      CSTF_TRY(admm_run(a, comm, st, nullptr, &iters, nullptr));
+      if (rep && rep->admm_iters) rep->admm_iters[t * N + n] = iters;
+      tm.end(n, CSTF_PHASE_UPDATE);
+      // a7: Gram of the update (raw), a6: lambda + normalisation (G scaled consistently)
+      tm.begin(n, CSTF_PHASE_GRAM);
+      CSTF_TRY(gram_raw(d_factors[n], I, R, Gn, st));
+      tm.end(n, CSTF_PHASE_GRAM);
+      tm.begin(n, CSTF_PHASE_NORMALIZE);
+      CSTF_TRY(normalize_from_gram(d_factors[n], I, R, Gn, lam + n * R, st));
+      tm.end(n, CSTF_PHASE_NORMALIZE);
+    }
+    // a8: fit of [[lambda^(N); H]] with M of the last mode
+    tm.begin(N - 1, CSTF_PHASE_NORMALIZE);
+    double* fb = w.fitbuf.as<double>();
+    CSTF_TRY(fit(X->normX2, X->dims[N - 1], R, M, d_factors[N - 1], lam + (N - 1) * R, G, N, fb + 4,
+                 fb, flag, comm, st));
+    tm.end(N - 1, CSTF_PHASE_NORMALIZE);
+    CSTF_CUDA(cudaMemcpyAsync(w.host_small, fb, 8, cudaMemcpyDeviceToHost, st));
+    CSTF_TRY(check_flag(flag, st));   // synchronises
+    tm.collect();
+    const double f = w.host_small[0];
+    if (rep) {
+      if (rep->fit) rep->fit[t] = f;
+      rep->outer_done = t + 1;
+    }
+    if (o->fit_tol > 0.0 && t > 0 && std::fabs(f - fit_prev) < o->fit_tol) break;
+    fit_prev = f;
+  }
+  if (d_lambda)
+    CSTF_CUDA(cudaMemcpyAsync(d_lambda, lam + (N - 1) * R, (size_t)R * 8, cudaMemcpyDeviceToDevice, st));
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  return CSTF_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+cstf_status cstf_tensor_load_coo(int nmodes, const int64_t* dims, int64_t nnz,
+                                 const int32_t* const* host_idx, const double* host_vals,
+                                 const cstf_comm* comm, void* stream, cstf_tensor** out) {
+  if (!out) return fail(CSTF_ERR_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (nmodes < 2 || nmodes > 8) return fail(CSTF_ERR_INVALID_ARG, "nmodes must be in [2, 8]");
+  if (!dims || nnz < 0) return fail(CSTF_ERR_INVALID_ARG, "dims NULL or nnz < 0");
+  if (nnz >= (int64_t)1 << 32) return fail(CSTF_ERR_UNSUPPORTED, "nnz >= 2^32");
+  if (nnz > 0 && (!host_idx || !host_vals)) return fail(CSTF_ERR_INVALID_ARG, "host arrays NULL");
+  for (int n = 0; n < nmodes; n++) {
+    if (dims[n] < 1 || dims[n] > 2147483647LL) return fail(CSTF_ERR_INVALID_ARG, "dims[n] must be in [1, 2^31-1]");
+    if (nnz > 0 && !host_idx[n]) return fail(CSTF_ERR_INVALID_ARG, "host_idx[n] is NULL");
+  }
+  if (comm_nranks(comm) > 1) return fail(CSTF_ERR_UNSUPPORTED, "partitioned load not built yet");
+  cstf_tensor* X = new cstf_tensor();
+  X->N = nmodes;
+  for (int n = 0; n < nmodes; n++) X->dims[n] = dims[n];
+  cudaGetDevice(&X->device);
+  cstf_status s = build_store(X, host_idx, host_vals, nnz, S(stream));
+  if (s != CSTF_OK) { delete X; return s; }
+  *out = X;
+  return CSTF_OK;
+}
+
+cstf_status cstf_tensor_info(const cstf_tensor* X, int* nmodes, int64_t* dims, int64_t* nnz_coalesced,
+                             double* normX2, uint64_t* canonical_hash) {
+  if (!X) return fail(CSTF_ERR_INVALID_ARG, "tensor is NULL");
+  if (nmodes) *nmodes = X->N;
+  if (dims) for (int n = 0; n < X->N; n++) dims[n] = X->dims[n];
+  if (nnz_coalesced) *nnz_coalesced = X->nnz;
+  if (normX2) *normX2 = X->normX2;
+  if (canonical_hash) *canonical_hash = X->hash;
+  return CSTF_OK;
+}
+
+cstf_status cstf_tensor_export_coo(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals) {
+  if (!X || (X->nnz > 0 && (!host_idx || !host_vals))) return fail(CSTF_ERR_INVALID_ARG, "export arguments");
+  if (X->nranks > 1) return fail(CSTF_ERR_UNSUPPORTED, "export of a partitioned tensor");
+  return export_store(X, host_idx, host_vals);
+}
+
+void cstf_tensor_free(cstf_tensor* X) { delete X; }
+
+cstf_status cstf_mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d_factors, double* d_M,
+                        void* stream) {
+  if (!X || !d_factors || !d_M) return fail(CSTF_ERR_INVALID_ARG, "NULL argument");
+  if (mode < 0 || mode >= X->N) return fail(CSTF_ERR_INVALID_ARG, "mode out of range");
+  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  for (int k = 0; k < X->N; k++)
+    if (k != mode && !d_factors[k]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");
+  return mttkrp(X, mode, R, d_factors, d_M, S(stream), nullptr);
+}
+
+cstf_status cstf_gram(const double* d_H, int64_t I, int R, double* d_G, const cstf_comm* comm, void* stream) {
+  if ((!d_H && I > 0) || !d_G || I < 0) return fail(CSTF_ERR_INVALID_ARG, "NULL argument or I < 0");
+  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  return gram_normalize(const_cast<double*>(d_H), I, R, d_G, nullptr, comm, S(stream), nullptr);
+}
+
+cstf_status cstf_normalize(double* d_H, int64_t I, int R, double* d_lambda, double* d_G, const cstf_comm* comm,
+                           void* stream) {
+  if ((!d_H && I > 0) || !d_lambda || I < 0) return fail(CSTF_ERR_INVALID_ARG, "NULL argument or I < 0");
+  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  DevBuf tmp;
+  double* G = d_G;
+  if (!G) { CSTF_TRY(tmp.alloc((size_t)R * R * 8)); G = tmp.as<double>(); }
+  CSTF_TRY(gram_normalize(d_H, I, R, G, d_lambda, comm, S(stream), nullptr));
+  if (!d_G) CSTF_CUDA(cudaStreamSynchronize(S(stream)));
+  return CSTF_OK;
+}
+
+cstf_status cstf_admm_update(const double* d_M, const double* d_S, double* d_H, double* d_U, int64_t I, int R,
+                             const cstf_admm_opts* opts, const cstf_comm* comm, cstf_admm_stats* host_stats,
+                             void* stream) {
+  if (!opts || !d_S || I < 0 || (I > 0 && (!d_M || !d_H || !d_U)))
+    return fail(CSTF_ERR_INVALID_ARG, "NULL argument or I < 0");
+  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  if (opts->max_iter < 1 || opts->tol < 0.0) return fail(CSTF_ERR_INVALID_ARG, "max_iter < 1 or tol < 0");
+  if (opts->prox != CSTF_PROX_NONNEG && opts->prox != CSTF_PROX_IDENTITY)
+    return fail(CSTF_ERR_INVALID_ARG, "unknown prox");
+  cudaStream_t st = S(stream);
+  DriverWs& w = dws();
+  CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
+  CSTF_TRY(w.scal.ensure(64));
+  CSTF_TRY(w.flag.ensure(64));
+  int* flag = w.flag.as<int>();
+  CSTF_CUDA(cudaMemsetAsync(flag, 0, 4, st));
+  CSTF_TRY(chol_inverse(d_S, nullptr, 0, -1, R, opts->rho, w.inv.as<double>(), w.scal.as<double>(), flag, st));
+  AdmmArgs a;
+  a.M = d_M; a.H = d_H; a.U = d_U; a.hscale = nullptr; a.I = I; a.R = R;
+  a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
+  a.tol = opts->tol; a.max_iter = opts->max_iter; a.prox = opts->prox; a.variant = opts->variant;
+  cstf_admm_stats stats;
+  CSTF_TRY(admm_run(a, comm, st, &stats, nullptr, nullptr));
+  CSTF_TRY(check_flag(flag, st));
+  if (host_stats) *host_stats = stats;
+  return CSTF_OK;
+}
+
+cstf_status cstf_factorize(const cstf_tensor* X, const cstf_opts* opts, const cstf_comm* comm,
+                           double* const* d_factors, double* d_lambda, cstf_report* report, void* stream) {
+  if (!X || !opts || !d_factors) return fail(CSTF_ERR_INVALID_ARG, "NULL argument");
+  return factorize_impl(X, opts, comm, d_factors, d_lambda, report, S(stream));
+}
+
+cstf_status cstf_factorize_host(const cstf_tensor* X, const cstf_opts* opts, const cstf_comm* comm,
+                                double* const* host_factors, double* host_lambda, cstf_report* report,
+                                void* stream) {
+  if (!X || !opts || !host_factors) return fail(CSTF_ERR_INVALID_ARG, "NULL argument");
+  if (!rank_ok(opts->R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  cudaStream_t st = S(stream);
+  DriverWs& w = dws();
+  const int N = X->N, R = opts->R;
+  int64_t tot = 0;
+  for (int n = 0; n < N; n++) tot += X->dims[n] * R;
+  CSTF_TRY(w.hostfac.ensure((size_t)(tot + R) * 8));
+  std::vector<double*> d(N);
+  int64_t off = 0;
+  for (int n = 0; n < N; n++) {
+    if (!host_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "host factor pointer is NULL");
+    d[n] = w.hostfac.as<double>() + off;
+    CSTF_CUDA(cudaMemcpyAsync(d[n], host_factors[n], (size_t)X->dims[n] * R * 8, cudaMemcpyHostToDevice, st));
+    off += X->dims[n] * R;
+  }
+  double* d_lam = w.hostfac.as<double>() + off;
+  CSTF_TRY(factorize_impl(X, opts, comm, d.data(), d_lam, report, st));
+  for (int n = 0; n < N; n++)
+    CSTF_CUDA(cudaMemcpyAsync(host_factors[n], d[n], (size_t)X->dims[n] * R * 8, cudaMemcpyDeviceToHost, st));
+  if (host_lambda) CSTF_CUDA(cudaMemcpyAsync(host_lambda, d_lam, (size_t)R * 8, cudaMemcpyDeviceToHost, st));
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  return CSTF_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,171 @@
+// Internal declarations of libcstf (host C++ / CUDA, sm_100a).  Not part of the ABI.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/cstf.h"
+
+namespace cstf {
+
+// ---------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+cstf_status fail(cstf_status s, const std::string& msg);
+cstf_status cuda_fail(cudaError_t e, const char* what);
+
+#define CSTF_CUDA(call)                                          \
+  do {                                                           \
+    cudaError_t e_ = (call);                                     \
+    if (e_ != cudaSuccess) return ::cstf::cuda_fail(e_, #call);  \
+  } while (0)
+#define CSTF_TRY(call)                         \
+  do {                                         \
+    cstf_status s_ = (call);                   \
+    if (s_ != CSTF_OK) return s_;              \
+  } while (0)
+// after a kernel launch
+#define CSTF_LAUNCHED() \
+  do { ::cstf::count_launch(); CSTF_CUDA(cudaGetLastError()); } while (0)
+
+void count_launch(int n = 1);
+
+// ---------------------------------------------------------------- device info
+struct DeviceInfo {
+  int device = -1;
+  int sms = 0;
+  size_t l2 = 0;
+  int max_smem_optin = 0;
+};
+const DeviceInfo& device_info();
+
+// ---------------------------------------------------------------- buffers
+// Owned device allocation (cudaMalloc / cudaFree).
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+  DevBuf() = default;
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  DevBuf(DevBuf&& o) noexcept : p(o.p), bytes(o.bytes) { o.p = nullptr; o.bytes = 0; }
+  DevBuf& operator=(DevBuf&& o) noexcept {
+    if (this != &o) { release(); p = o.p; bytes = o.bytes; o.p = nullptr; o.bytes = 0; }
+    return *this;
+  }
+  ~DevBuf() { release(); }
+  void release();
+  cstf_status alloc(size_t n);          // exact (re)allocation, contents undefined
+  cstf_status ensure(size_t n);         // grow-only
+  template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+// Grow-only scratch arena carved into aligned slices.
+struct Arena {
+  DevBuf buf;
+  size_t used = 0;
+  std::vector<size_t> pending;  // requested sizes while planning
+  void reset() { used = 0; }
+  // returns aligned pointer inside buf (caller must have ensured capacity)
+  void* take(size_t n);
+};
+
+// ---------------------------------------------------------------- comm
+struct Comm {
+  int nranks = 1;
+  int rank = 0;
+  void* nccl = nullptr;  // ncclComm_t
+};
+cstf_status comm_allreduce_f64(const cstf_comm* c, double* d_buf, size_t count, cudaStream_t st);
+cstf_status comm_allgather_f64(const cstf_comm* c, const double* d_send, double* d_recv,
+                               size_t count_per_rank, cudaStream_t st);
+int comm_nranks(const cstf_comm* c);
+int comm_rank(const cstf_comm* c);
+
+// ---------------------------------------------------------------- tensor store
+struct ModeStore {
+  int64_t I = 0;            // rows of this mode (local rows when distributed)
+  int64_t nnz = 0;          // nonzeros in this copy
+  DevBuf rowptr;            // int64[I+1]
+  DevBuf idx[7];            // int32[nnz] for the other modes (increasing mode order)
+  DevBuf vals;              // double[nnz]
+  int other[7];             // mode id of idx[k]
+};
+
+}  // namespace cstf
+
+struct cstf_comm {
+  cstf::Comm c;
+};
+
+struct cstf_tensor {
+  int N = 0;
+  int64_t dims[8] = {0};
+  int64_t nnz = 0;          // coalesced (local share when distributed)
+  double normX2 = 0.0;
+  uint64_t hash = 0;
+  int device = -1;
+  cstf::ModeStore mode[8];
+  // distributed layout (nranks > 1): relabel maps original -> internal label
+  int nranks = 1, rank = 0;
+  int64_t rows_per_rank[8] = {0};     // block size per rank (padded), per mode
+  cstf::DevBuf relabel[8];            // int32[dims[n]]: internal label of original row
+  cstf::DevBuf unlabel[8];            // int32[nranks*rows_per_rank]: original row (or -1 pad)
+};
+
+namespace cstf {
+
+// ---------------------------------------------------------------- kernels (launchers)
+// store.cu
+cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const double* host_vals,
+                        int64_t nnz_in, cudaStream_t st);
+cstf_status export_store(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals);
+
+// mttkrp.cu
+cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d_factors,
+                   double* d_M, cudaStream_t st, int64_t* launches);
+
+// dense.cu
+// G (R x R) = H^T H; if lam != nullptr also normalises: lam_r = sqrt(G_rr), H /= lam (in place),
+// G <- D^-1 G D^-1.  comm: all-reduce the raw Gram.
+cstf_status gram_normalize(double* d_H, int64_t I, int R, double* d_G, double* d_lam,
+                           const cstf_comm* comm, cudaStream_t st, int64_t* launches);
+// pieces of gram_normalize (no comm): raw Gram, then lam / G scaling / H /= lam
+cstf_status gram_raw(const double* d_H, int64_t I, int R, double* d_G, cudaStream_t st);
+cstf_status normalize_from_gram(double* d_H, int64_t I, int R, double* d_G, double* d_lam,
+                                cudaStream_t st);
+cstf_status fill(double* d, int64_t n, double v, cudaStream_t st);
+// One CTA: S = Hadamard of the Grams except `skip` (or copy of d_S when grams == nullptr),
+// rho, Cholesky of S + rho I, Inv = (S + rho I)^-1.  Writes d_inv (R x R), d_scal[0] = rho,
+// d_flag |= 1 on NOT_SPD.
+cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int skip, int R,
+                         double rho_in, double* d_inv, double* d_scal, int* d_flag,
+                         cudaStream_t st);
+// fit (D12): writes d_out[0] = fit; needs M of the last mode, its H, lam, all Grams.
+cstf_status fit(double normX2, int64_t I, int R, const double* d_M, const double* d_H,
+                const double* d_lam, const double* d_grams, int N, double* d_part /* >= 256 */,
+                double* d_out /* [2] */, int* d_flag, const cstf_comm* comm, cudaStream_t st);
+cstf_status scale_rows_by_cols(double* d_H, int64_t I, int R, const double* d_lam, int divide,
+                               cudaStream_t st);
+
+// admm.cu
+struct AdmmArgs {
+  const double* M;
+  double* H;
+  double* U;
+  const double* hscale;  // optional per-column scale of the incoming H (warm start D4)
+  int64_t I;
+  int R;
+  const double* inv;     // device R x R
+  const double* scal;    // device: [0] = rho
+  int* flag;             // device status flags
+  double tol;
+  int max_iter;
+  int prox;
+  int variant;
+};
+cstf_status admm_run(const AdmmArgs& a, const cstf_comm* comm, cudaStream_t st,
+                     cstf_admm_stats* stats, int* iters_out, int64_t* launches);
+
+}  // namespace cstf

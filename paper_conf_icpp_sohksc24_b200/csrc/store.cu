@@ -1,0 +1,408 @@
+// Mode-sorted nonzero store (hot-path step a0).
+//
+// Host COO -> device -> validate -> canonical order (lexicographic by
+// (i_1..i_N), LSD radix sort over <=64-bit packed mode groups, stable so
+// duplicates keep input order) -> duplicates summed left to right in input
+// order (bit-exact with the oracle's O1) -> ||X||^2 and canonical checksum ->
+// for every mode n a copy stably sorted by i_n with an int64 row pointer.
+// The element-wise MTTKRP definition this store serves is PAPER.md Fig. 2
+// (L403-430); the paper's own format (BLCO, L439-442) is replaced.
+#include <cub/cub.cuh>
+
+#include <cstring>
+
+#include "internal.h"
+
+namespace cstf {
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kFixedBlocks = 1024;  // fixed => deterministic reductions
+
+inline int grid_for(int64_t n, int threads = kThreads) {
+  int64_t g = (n + threads - 1) / threads;
+  int cap = device_info().sms * 32;
+  if (g > cap) g = cap;
+  return (int)(g < 1 ? 1 : g);
+}
+
+int bits_for(int64_t dim) {
+  int b = 0;
+  while (b < 63 && ((int64_t)1 << b) < dim) b++;
+  return b;  // dim == 1 -> 0 bits
+}
+
+__global__ void k_count_invalid(const int32_t* __restrict__ idx, int64_t n, int64_t dim,
+                                unsigned long long* bad) {
+  unsigned long long c = 0;
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    int32_t v = idx[p];
+    c += (v < 0 || (int64_t)v >= dim) ? 1ull : 0ull;
+  }
+  if (c) atomicAdd(bad, c);
+}
+
+struct PackArgs {
+  const int32_t* idx[8];
+  int shift[8];
+  int count;
+};
+
+// key[p] = packed indices of the group's modes for the nonzero perm[p] (or p when perm == null)
+__global__ void k_pack_keys(PackArgs a, const uint32_t* __restrict__ perm, int64_t n,
+                            uint64_t* __restrict__ key) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    uint64_t src = perm ? perm[p] : (uint64_t)p;
+    uint64_t k = 0;
+    for (int m = 0; m < a.count; m++) k |= (uint64_t)(uint32_t)a.idx[m][src] << a.shift[m];
+    key[p] = k;
+  }
+}
+
+__global__ void k_iota(uint32_t* __restrict__ out, int64_t n) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    out[p] = (uint32_t)p;
+}
+
+template <class T>
+__global__ void k_gather(const T* __restrict__ in, const uint32_t* __restrict__ perm, int64_t n,
+                         T* __restrict__ out) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    out[p] = in[perm[p]];
+}
+
+struct IdxArgs {
+  const int32_t* idx[8];
+  int N;
+};
+
+__global__ void k_heads(IdxArgs a, int64_t n, uint32_t* __restrict__ head) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    uint32_t h = (p == 0);
+    if (!h)
+      for (int m = 0; m < a.N; m++) h |= (a.idx[m][p] != a.idx[m][p - 1]);
+    head[p] = h;
+  }
+}
+
+// segid = inclusive scan of heads (1-based); start[segid-1] = p at heads
+__global__ void k_seg_starts(const uint32_t* __restrict__ head, const uint32_t* __restrict__ segid,
+                             int64_t n, uint32_t* __restrict__ start) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    if (head[p]) start[segid[p] - 1] = (uint32_t)p;
+}
+
+struct OutArgs {
+  int32_t* idx[8];
+  int N;
+};
+
+// one thread per coalesced entry: left-to-right sum of the duplicates (input order)
+__global__ void k_coalesce(IdxArgs in, const double* __restrict__ vals,
+                           const uint32_t* __restrict__ start, int64_t nseg, int64_t n,
+                           OutArgs out, double* __restrict__ out_vals) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < nseg;
+       s += (int64_t)gridDim.x * blockDim.x) {
+    int64_t p0 = start[s];
+    int64_t p1 = (s + 1 < nseg) ? (int64_t)start[s + 1] : n;
+    double v = vals[p0];
+    for (int64_t p = p0 + 1; p < p1; p++) v = __dadd_rn(v, vals[p]);
+    out_vals[s] = v;
+    for (int m = 0; m < in.N; m++) out.idx[m][s] = in.idx[m][p0];
+  }
+}
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+  z ^= z >> 30; z *= 0xBF58476D1CE4E5B9ULL;
+  z ^= z >> 27; z *= 0x94D049BB133111EBULL;
+  z ^= z >> 31; return z;
+}
+
+// Per fixed block: partial sum of v^2 (tree order) and of the entry checksums (mod 2^64).
+__global__ void __launch_bounds__(kThreads) k_norm_hash(IdxArgs a, const double* __restrict__ vals,
+                                                        int64_t n, double* __restrict__ part_norm,
+                                                        unsigned long long* __restrict__ part_hash) {
+  __shared__ double sn[kThreads];
+  __shared__ unsigned long long sh[kThreads];
+  double acc = 0.0;
+  unsigned long long h = 0;
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    double v = vals[p];
+    acc = fma(v, v, acc);
+    uint64_t z = (uint64_t)p + 1;
+    for (int m = 0; m < a.N; m++)
+      z = mix64(z ^ ((uint64_t)(uint32_t)a.idx[m][p] + (uint64_t)(m + 1) * 0x9E3779B97F4A7C15ULL));
+    z = mix64(z ^ (uint64_t)__double_as_longlong(v));
+    h += z;
+  }
+  sn[threadIdx.x] = acc;
+  sh[threadIdx.x] = h;
+  __syncthreads();
+  for (int s = kThreads / 2; s > 0; s >>= 1) {
+    if (threadIdx.x < s) {
+      sn[threadIdx.x] += sn[threadIdx.x + s];
+      sh[threadIdx.x] += sh[threadIdx.x + s];
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    part_norm[blockIdx.x] = sn[0];
+    part_hash[blockIdx.x] = sh[0];
+  }
+}
+
+__global__ void k_norm_hash_final(const double* __restrict__ part_norm,
+                                  const unsigned long long* __restrict__ part_hash, int nb,
+                                  double* out_norm, unsigned long long* out_hash) {
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    double s = 0.0;
+    unsigned long long h = 0;
+    for (int b = 0; b < nb; b++) { s += part_norm[b]; h += part_hash[b]; }
+    *out_norm = s;
+    *out_hash = h;
+  }
+}
+
+__global__ void k_histogram(const int32_t* __restrict__ key, int64_t n,
+                            unsigned long long* __restrict__ cnt) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(&cnt[key[p]], 1ull);
+}
+
+__global__ void k_expand_rows(const int64_t* __restrict__ rowptr, int64_t I,
+                              int32_t* __restrict__ out) {
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < I;
+       i += (int64_t)gridDim.x * blockDim.x)
+    for (int64_t p = rowptr[i]; p < rowptr[i + 1]; p++) out[p] = (int32_t)i;
+}
+
+// rowptr[0] = 0, rowptr[i+1] = sum_{r<=i} counts[r]
+cstf_status build_rowptr(const int32_t* d_key, int64_t n, int64_t I, DevBuf& rowptr, DevBuf& tmp,
+                         cudaStream_t st) {
+  CSTF_TRY(rowptr.alloc((size_t)(I + 1) * 8));
+  DevBuf cnt;
+  CSTF_TRY(cnt.alloc((size_t)I * 8));
+  CSTF_CUDA(cudaMemsetAsync(cnt.p, 0, (size_t)I * 8, st));
+  CSTF_CUDA(cudaMemsetAsync(rowptr.p, 0, 8, st));
+  if (n > 0) {
+    k_histogram<<<grid_for(n), kThreads, 0, st>>>(d_key, n, cnt.as<unsigned long long>());
+    CSTF_LAUNCHED();
+  }
+  size_t tb = 0;
+  CSTF_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, cnt.as<unsigned long long>(),
+                                          (unsigned long long*)(rowptr.as<int64_t>() + 1), I, st));
+  CSTF_TRY(tmp.ensure(tb));
+  CSTF_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, tb, cnt.as<unsigned long long>(),
+                                          (unsigned long long*)(rowptr.as<int64_t>() + 1), I, st));
+  count_launch();
+  CSTF_CUDA(cudaStreamSynchronize(st));  // cnt freed on return
+  return CSTF_OK;
+}
+
+}  // namespace
+
+cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const double* host_vals,
+                        int64_t n, cudaStream_t st) {
+  const int N = X->N;
+  DevBuf tmp;  // cub temp storage
+  // ---- 1. upload + validate
+  DevBuf in_idx[8], in_vals;
+  for (int m = 0; m < N; m++) {
+    CSTF_TRY(in_idx[m].alloc((size_t)n * 4));
+    if (n) CSTF_CUDA(cudaMemcpyAsync(in_idx[m].p, host_idx[m], (size_t)n * 4, cudaMemcpyHostToDevice, st));
+  }
+  CSTF_TRY(in_vals.alloc((size_t)n * 8));
+  if (n) CSTF_CUDA(cudaMemcpyAsync(in_vals.p, host_vals, (size_t)n * 8, cudaMemcpyHostToDevice, st));
+  {
+    DevBuf bad;
+    CSTF_TRY(bad.alloc(8));
+    CSTF_CUDA(cudaMemsetAsync(bad.p, 0, 8, st));
+    for (int m = 0; m < N && n > 0; m++) {
+      k_count_invalid<<<grid_for(n), kThreads, 0, st>>>(in_idx[m].as<int32_t>(), n, X->dims[m],
+                                                        bad.as<unsigned long long>());
+      CSTF_LAUNCHED();
+    }
+    unsigned long long nbad = 0;
+    CSTF_CUDA(cudaMemcpyAsync(&nbad, bad.p, 8, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    if (nbad) return fail(CSTF_ERR_INVALID_ARG, std::to_string(nbad) + " indices outside [0, dims[n])");
+  }
+  // ---- 2. canonical order: LSD radix sort over packed groups of modes, last group first
+  DevBuf perm_a, perm_b, key_a, key_b;
+  CSTF_TRY(perm_a.alloc((size_t)n * 4));
+  CSTF_TRY(perm_b.alloc((size_t)n * 4));
+  CSTF_TRY(key_a.alloc((size_t)n * 8));
+  CSTF_TRY(key_b.alloc((size_t)n * 8));
+  if (n) {
+    k_iota<<<grid_for(n), kThreads, 0, st>>>(perm_a.as<uint32_t>(), n);
+    CSTF_LAUNCHED();
+  }
+  int hi = N - 1;
+  while (hi >= 0 && n > 0) {
+    // group = modes [lo, hi] with total bits <= 64
+    int lo = hi, tot = bits_for(X->dims[hi]);
+    while (lo - 1 >= 0 && tot + bits_for(X->dims[lo - 1]) <= 64) { lo--; tot += bits_for(X->dims[lo]); }
+    PackArgs pa;
+    pa.count = hi - lo + 1;
+    int sh = 0;
+    for (int m = hi; m >= lo; m--) {  // lowest mode most significant
+      pa.idx[m - lo] = in_idx[m].as<int32_t>();
+      pa.shift[m - lo] = sh;
+      sh += bits_for(X->dims[m]);
+    }
+    if (tot > 0) {
+      k_pack_keys<<<grid_for(n), kThreads, 0, st>>>(pa, perm_a.as<uint32_t>(), n, key_a.as<uint64_t>());
+      CSTF_LAUNCHED();
+      size_t tb = 0;
+      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, key_a.as<uint64_t>(), key_b.as<uint64_t>(),
+                                                perm_a.as<uint32_t>(), perm_b.as<uint32_t>(), n, 0, tot, st));
+      CSTF_TRY(tmp.ensure(tb));
+      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, key_a.as<uint64_t>(), key_b.as<uint64_t>(),
+                                                perm_a.as<uint32_t>(), perm_b.as<uint32_t>(), n, 0, tot, st));
+      count_launch();
+      std::swap(perm_a, perm_b);
+    }
+    hi = lo - 1;
+  }
+  key_a.release(); key_b.release(); perm_b.release();
+  // ---- 3. gather into sorted order, free the inputs
+  DevBuf s_idx[8], s_vals;
+  for (int m = 0; m < N; m++) {
+    CSTF_TRY(s_idx[m].alloc((size_t)n * 4));
+    if (n) { k_gather<int32_t><<<grid_for(n), kThreads, 0, st>>>(in_idx[m].as<int32_t>(), perm_a.as<uint32_t>(), n, s_idx[m].as<int32_t>()); CSTF_LAUNCHED(); }
+  }
+  CSTF_TRY(s_vals.alloc((size_t)n * 8));
+  if (n) { k_gather<double><<<grid_for(n), kThreads, 0, st>>>(in_vals.as<double>(), perm_a.as<uint32_t>(), n, s_vals.as<double>()); CSTF_LAUNCHED(); }
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  for (int m = 0; m < N; m++) in_idx[m].release();
+  in_vals.release();
+  // ---- 4. duplicates: heads, segment ids, left-to-right sums
+  IdxArgs sa;
+  sa.N = N;
+  for (int m = 0; m < N; m++) sa.idx[m] = s_idx[m].as<int32_t>();
+  int64_t nout = 0;
+  DevBuf c_idx[8], c_vals;
+  {
+    DevBuf head, segid;
+    CSTF_TRY(head.alloc((size_t)n * 4));
+    CSTF_TRY(segid.alloc((size_t)n * 4));
+    if (n) {
+      k_heads<<<grid_for(n), kThreads, 0, st>>>(sa, n, head.as<uint32_t>());
+      CSTF_LAUNCHED();
+      size_t tb = 0;
+      CSTF_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, head.as<uint32_t>(), segid.as<uint32_t>(), n, st));
+      CSTF_TRY(tmp.ensure(tb));
+      CSTF_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, tb, head.as<uint32_t>(), segid.as<uint32_t>(), n, st));
+      count_launch();
+      uint32_t last = 0;
+      CSTF_CUDA(cudaMemcpyAsync(&last, segid.as<uint32_t>() + n - 1, 4, cudaMemcpyDeviceToHost, st));
+      CSTF_CUDA(cudaStreamSynchronize(st));
+      nout = last;
+    }
+    // reuse perm_a as segment starts
+    if (n) { k_seg_starts<<<grid_for(n), kThreads, 0, st>>>(head.as<uint32_t>(), segid.as<uint32_t>(), n, perm_a.as<uint32_t>()); CSTF_LAUNCHED(); }
+    OutArgs oa;
+    oa.N = N;
+    for (int m = 0; m < N; m++) {
+      CSTF_TRY(c_idx[m].alloc((size_t)nout * 4));
+      oa.idx[m] = c_idx[m].as<int32_t>();
+    }
+    CSTF_TRY(c_vals.alloc((size_t)nout * 8));
+    if (nout) {
+      k_coalesce<<<grid_for(nout), kThreads, 0, st>>>(sa, s_vals.as<double>(), perm_a.as<uint32_t>(), nout, n, oa, c_vals.as<double>());
+      CSTF_LAUNCHED();
+    }
+    CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  for (int m = 0; m < N; m++) s_idx[m].release();
+  s_vals.release();
+  perm_a.release();
+  X->nnz = nout;
+  // ---- 5. ||X||^2 and checksum (fixed grid => deterministic)
+  {
+    IdxArgs ca;
+    ca.N = N;
+    for (int m = 0; m < N; m++) ca.idx[m] = c_idx[m].as<int32_t>();
+    DevBuf pn, ph, out;
+    CSTF_TRY(pn.alloc(kFixedBlocks * 8));
+    CSTF_TRY(ph.alloc(kFixedBlocks * 8));
+    CSTF_TRY(out.alloc(16));
+    k_norm_hash<<<kFixedBlocks, kThreads, 0, st>>>(ca, c_vals.as<double>(), nout, pn.as<double>(), ph.as<unsigned long long>());
+    CSTF_LAUNCHED();
+    k_norm_hash_final<<<1, 32, 0, st>>>(pn.as<double>(), ph.as<unsigned long long>(), kFixedBlocks, out.as<double>(), (unsigned long long*)(out.as<double>() + 1));
+    CSTF_LAUNCHED();
+    double hv[2];
+    CSTF_CUDA(cudaMemcpyAsync(hv, out.p, 16, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    X->normX2 = hv[0];
+    memcpy(&X->hash, &hv[1], 8);
+  }
+  // ---- 6. per-mode copies, stably sorted by i_n (mode 0 = canonical order)
+  for (int n_ = N - 1; n_ >= 0; n_--) {
+    ModeStore& ms = X->mode[n_];
+    ms.I = X->dims[n_];
+    ms.nnz = nout;
+    int k = 0;
+    for (int m = 0; m < N; m++)
+      if (m != n_) ms.other[k++] = m;
+    if (n_ == 0) {
+      CSTF_TRY(build_rowptr(c_idx[0].as<int32_t>(), nout, ms.I, ms.rowptr, tmp, st));
+      for (int q = 0; q < N - 1; q++) ms.idx[q] = std::move(c_idx[ms.other[q]]);
+      ms.vals = std::move(c_vals);
+      c_idx[0].release();
+      break;
+    }
+    DevBuf keys_out, pm_in, pm_out;
+    CSTF_TRY(keys_out.alloc((size_t)nout * 4));
+    CSTF_TRY(pm_in.alloc((size_t)nout * 4));
+    CSTF_TRY(pm_out.alloc((size_t)nout * 4));
+    if (nout) {
+      k_iota<<<grid_for(nout), kThreads, 0, st>>>(pm_in.as<uint32_t>(), nout);
+      CSTF_LAUNCHED();
+      int nb = bits_for(ms.I);
+      size_t tb = 0;
+      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const uint32_t*)c_idx[n_].p, keys_out.as<uint32_t>(),
+                                                pm_in.as<uint32_t>(), pm_out.as<uint32_t>(), nout, 0, nb > 0 ? nb : 1, st));
+      CSTF_TRY(tmp.ensure(tb));
+      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const uint32_t*)c_idx[n_].p, keys_out.as<uint32_t>(),
+                                                pm_in.as<uint32_t>(), pm_out.as<uint32_t>(), nout, 0, nb > 0 ? nb : 1, st));
+      count_launch();
+    }
+    CSTF_TRY(build_rowptr(keys_out.as<int32_t>(), nout, ms.I, ms.rowptr, tmp, st));
+    for (int q = 0; q < N - 1; q++) {
+      CSTF_TRY(ms.idx[q].alloc((size_t)nout * 4));
+      if (nout) { k_gather<int32_t><<<grid_for(nout), kThreads, 0, st>>>(c_idx[ms.other[q]].as<int32_t>(), pm_out.as<uint32_t>(), nout, ms.idx[q].as<int32_t>()); CSTF_LAUNCHED(); }
+    }
+    CSTF_TRY(ms.vals.alloc((size_t)nout * 8));
+    if (nout) { k_gather<double><<<grid_for(nout), kThreads, 0, st>>>(c_vals.as<double>(), pm_out.as<uint32_t>(), nout, ms.vals.as<double>()); CSTF_LAUNCHED(); }
+    CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  return CSTF_OK;
+}
+
+cstf_status export_store(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals) {
+  const ModeStore& ms = X->mode[0];
+  int64_t n = ms.nnz;
+  cudaStream_t st = 0;
+  if (n == 0) return CSTF_OK;
+  DevBuf rows;
+  CSTF_TRY(rows.alloc((size_t)n * 4));
+  k_expand_rows<<<grid_for(ms.I), kThreads, 0, st>>>(ms.rowptr.as<int64_t>(), ms.I, rows.as<int32_t>());
+  CSTF_LAUNCHED();
+  CSTF_CUDA(cudaMemcpy(host_idx[0], rows.p, (size_t)n * 4, cudaMemcpyDeviceToHost));
+  for (int q = 0; q < X->N - 1; q++)
+    CSTF_CUDA(cudaMemcpy(host_idx[ms.other[q]], ms.idx[q].p, (size_t)n * 4, cudaMemcpyDeviceToHost));
+  CSTF_CUDA(cudaMemcpy(host_vals, ms.vals.p, (size_t)n * 8, cudaMemcpyDeviceToHost));
+  return CSTF_OK;
+}
+
+}  // namespace cstf

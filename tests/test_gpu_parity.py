@@ -1,0 +1,313 @@
+"""GPU parity: the CUDA path (through the C ABI) against the FP64 oracle on the
+same seeded inputs.  Tolerances (north_star):
+  integer / index / order work ........ bit-exact (canonical order, checksum)
+  MTTKRP, fixed-iteration ADMM ........ normwise max rel <= 1e-9 (reading D18)
+  Gram / normalize ..................... <= 1e-12
+  end-to-end fit (10 outer iterations) . rel diff <= 1e-6, ADMM iteration counts equal
+"""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from parity_util import compare_iteration_counts
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-9
+
+
+@pytest.fixture(scope="module")
+def B():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_sohksc24_b200 import binding
+    return binding
+
+
+def normwise(a, b):
+    a = np.asarray(a, dtype=np.float64)
+    b = np.asarray(b, dtype=np.float64)
+    den = np.max(np.abs(b)) if b.size else 0.0
+    return float(np.max(np.abs(a - b)) / (den if den > 0 else 1.0)) if b.size else 0.0
+
+
+def cu(a):
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.float64)).cuda()
+
+
+def host(t):
+    torch.cuda.synchronize()
+    return t.cpu().numpy()
+
+
+def random_coo(seed, dims, nnz, dup_frac=0.2):
+    rng = np.random.default_rng(seed)
+    idx = [rng.integers(0, I, nnz).astype(np.int32) for I in dims]
+    nd = int(nnz * dup_frac)
+    if nd:
+        s, d = rng.integers(0, nnz, nd), rng.integers(0, nnz, nd)
+        for a in idx:
+            a[d] = a[s]
+    vals = rng.random(nnz) + 0.1
+    vals[rng.random(nnz) < 0.05] *= -1
+    vals[rng.random(nnz) < 0.02] = 0.0
+    return idx, vals
+
+
+STORE_CASES = [
+    ("3mode-dups", (40, 31, 17), 5000, 1),
+    ("4mode-dups", (9, 8, 7, 6), 3000, 2),
+    ("2mode", (100, 77), 2000, 3),
+    ("unit-dim", (1, 50, 1), 300, 4),
+    ("wide-keys", (2_000_000_000, 1_500_000_000, 1_000_000_000), 20000, 5),   # > 64 key bits
+]
+
+
+@pytest.mark.parametrize("name,dims,nnz,seed", STORE_CASES)
+def test_store_canonical_order_bit_exact(B, name, dims, nnz, seed):
+    idx, vals = random_coo(seed, dims, nnz, dup_frac=0.0 if name == "wide-keys" else 0.3)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    info = X.info()
+    assert info["nnz"] == ref.nnz
+    assert info["hash"] == ref.hash
+    gi, gv = X.export_coo()
+    for a, b in zip(gi, ref.idx):
+        assert np.array_equal(a, b)
+    assert np.array_equal(gv, ref.vals)                    # duplicates summed in input order
+    assert info["normX2"] == pytest.approx(ref.normX2, rel=1e-13)
+
+
+def test_store_empty_and_single(B):
+    X = B.cstf_tensor_load_coo((4, 5, 6), [np.zeros(0, np.int32)] * 3, np.zeros(0))
+    assert X.info()["nnz"] == 0
+    F = [cu(np.ones((I, 3))) for I in (4, 5, 6)]
+    M = cu(np.full((4, 3), 7.0))
+    B.cstf_mttkrp(X, 0, F, M)
+    assert np.all(host(M) == 0.0)
+    X1 = B.cstf_tensor_load_coo((4, 5, 6), [np.array([3], np.int32), np.array([1], np.int32), np.array([5], np.int32)],
+                                np.array([2.5]))
+    M = cu(np.zeros((4, 3)))
+    B.cstf_mttkrp(X1, 0, F, M)
+    assert np.array_equal(host(M), np.array([[0, 0, 0]] * 3 + [[2.5] * 3], dtype=float))
+
+
+def test_store_rejects_out_of_range(B):
+    with pytest.raises(B.CstfError) as e:
+        B.cstf_tensor_load_coo((3, 3), [np.array([0, 3], np.int32), np.array([0, 1], np.int32)], np.ones(2))
+    assert e.value.status == B.CSTF_ERR_INVALID_ARG
+
+
+MTTKRP_CASES = [
+    ((300, 200, 500), (2, 2, 3), 40000, 7),
+    ((60, 5000, 40, 30), (2, 3, 1, 2), 60000, 8),
+    ((1000, 900), (3, 1), 30000, 9),
+    ((50, 40, 30, 20, 10), (1, 2, 1, 2, 1), 8000, 10),
+]
+
+
+@pytest.mark.parametrize("case", MTTKRP_CASES)
+@pytest.mark.parametrize("R", [1, 5, 16, 32, 33, 64, 100, 128])
+def test_mttkrp_parity(B, case, R):
+    dims, gam, nnz, seed = case
+    idx, vals = datagen.coo(dims, gam, nnz, seed)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    F = datagen.init_factors(dims, R, seed)
+    Fd = [cu(f) for f in F]
+    for n in range(len(dims)):
+        M = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        want = oracle.mttkrp(ref, n, F)
+        assert normwise(host(M), want) <= TOL, (n, R)
+
+
+def test_mttkrp_heavy_row_spans_many_chunks(B):
+    """One row holding most nonzeros (carry fix-up across many chunks) + empty rows."""
+    rng = np.random.default_rng(3)
+    nnz = 300_000
+    i = np.where(rng.random(nnz) < 0.9, 7, rng.integers(0, 50, nnz)).astype(np.int32)
+    i[i == 3] = 4                                            # row 3 empty
+    j = rng.integers(0, 400, nnz).astype(np.int32)
+    k = rng.integers(0, 300, nnz).astype(np.int32)
+    dims = (50, 400, 300)
+    vals = rng.random(nnz)
+    X = B.cstf_tensor_load_coo(dims, [i, j, k], vals)
+    ref = oracle.coalesce(dims, [i, j, k], vals)
+    F = [rng.random((I, 32)) for I in dims]
+    M = cu(np.full((50, 32), np.nan))
+    B.cstf_mttkrp(X, 0, [cu(f) for f in F], M)
+    got = host(M)
+    assert np.all(got[3] == 0.0)
+    assert normwise(got, oracle.mttkrp(ref, 0, F)) <= TOL
+
+
+def test_mttkrp_deterministic(B):
+    dims = (300, 200, 500)
+    idx, vals = datagen.coo(dims, (2, 2, 3), 40000, 7)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    F = [cu(f) for f in datagen.init_factors(dims, 32, 7)]
+    outs = []
+    for _ in range(3):
+        M = cu(np.zeros((500, 32)))
+        B.cstf_mttkrp(X, 2, F, M)
+        outs.append(host(M))
+    assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[1], outs[2])
+
+
+@pytest.mark.parametrize("I,R", [(1, 4), (1000, 8), (4099, 32), (777, 64), (300, 100), (5000, 3)])
+def test_gram_and_normalize(B, I, R):
+    H = datagen.uniform(5, 77, I * R).reshape(I, R)
+    H[:, R // 2] = 0.0
+    G = cu(np.zeros((R, R)))
+    B.cstf_gram(cu(H), G)
+    assert normwise(host(G), oracle.gram(H)) <= 1e-12
+    Hd = cu(H)
+    lam = cu(np.zeros(R))
+    G2 = cu(np.zeros((R, R)))
+    B.cstf_normalize(Hd, lam, G2)
+    Hn, lam_ref = oracle.normalize(H)
+    assert normwise(host(lam), lam_ref) <= 1e-12
+    assert normwise(host(Hd), Hn) <= 1e-12
+    assert host(lam)[R // 2] == 0.0 and np.all(host(Hd)[:, R // 2] == 0.0)
+    assert normwise(host(G2), oracle.gram(Hn)) <= 1e-12
+
+
+def admm_inputs(I, R, seed, nmodes=3):
+    """M, S, H, U shaped like a real update: S = Hadamard of Grams of normalised factors."""
+    Fs = [oracle.normalize(datagen.uniform(seed, 10 + k, 200 * R).reshape(200, R))[0] for k in range(nmodes)]
+    S = oracle.hadamard_except([oracle.gram(F) for F in Fs], 0)
+    M = datagen.uniform(seed, 20, I * R).reshape(I, R) * 2.0 - 0.5
+    H = datagen.uniform(seed, 21, I * R).reshape(I, R)
+    U = (datagen.uniform(seed, 22, I * R).reshape(I, R) - 0.5) * 0.1
+    return M, S, H, U
+
+
+@pytest.mark.parametrize("variant", [0, 1, 2])
+@pytest.mark.parametrize("I,R", [(1, 8), (1003, 3), (4097, 8), (2049, 16), (3001, 32), (1500, 40), (999, 64),
+                                 (600, 65), (300, 128)])
+def test_admm_fixed_iterations(B, variant, I, R):
+    M, S, H, U = admm_inputs(I, R, R + I)
+    Hd, Ud = cu(H), cu(U)
+    st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=0.0, max_iter=10, variant=variant)
+    Hr, Ur, sr = oracle.admm(M, S, H, U, tol=0.0, max_iter=10)
+    assert st["iters"] == sr["iters"] == 10
+    assert normwise(host(Hd), Hr) <= TOL
+    assert normwise(host(Ud), Ur) <= TOL
+    for k in ("rho", "r_primal", "s_dual", "normH2", "normU2"):
+        assert st[k] == pytest.approx(sr[k], rel=1e-9, abs=1e-300), k
+
+
+@pytest.mark.parametrize("max_iter", [1, 17, 40])
+def test_admm_iteration_chunking(B, max_iter):
+    M, S, H, U = admm_inputs(2000, 32, 5)
+    Hd, Ud = cu(H), cu(U)
+    B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=0.0, max_iter=max_iter)
+    Hr, Ur, _ = oracle.admm(M, S, H, U, tol=0.0, max_iter=max_iter)
+    assert normwise(host(Hd), Hr) <= TOL and normwise(host(Ud), Ur) <= TOL
+
+
+def stop_margin(trace, j, eps):
+    r, s, nH, nU = trace[j]
+    return min(eps * nH - r, eps * nU - s) / (eps * (nH + nU))
+
+
+@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("eps,R", [(1e-1, 16), (1e-2, 32), (1e-3, 32), (1e-2, 64), (1e-2, 100)])
+def test_admm_tolerance_mode(B, variant, eps, R):
+    """Iteration count parity with the oracle's stopping rule (D3); U2 margin logged."""
+    M, S, H, U = admm_inputs(3000, R, 99)
+    Hd, Ud = cu(H), cu(U)
+    st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=eps, max_iter=30, variant=variant)
+    Hr, Ur, sr, tr = oracle.admm(M, S, H, U, tol=eps, max_iter=30, trace=True)
+    if st["iters"] != sr["iters"]:
+        j = min(st["iters"], sr["iters"]) - 1
+        assert abs(stop_margin(tr, j, eps)) < 1e-12, "iteration counts differ away from a tie"
+        pytest.skip("tie at the decisive iteration (U2)")
+    assert normwise(host(Hd), Hr) <= TOL and normwise(host(Ud), Ur) <= TOL
+
+
+def test_admm_identity_prox(B):
+    M, S, H, U = admm_inputs(500, 16, 3)
+    Hd, Ud = cu(H), cu(U)
+    B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=0.0, max_iter=12, prox=B.CSTF_PROX_IDENTITY)
+    Hr, Ur, _ = oracle.admm(M, S, H, U, tol=0.0, max_iter=12, prox=oracle.PROX_IDENTITY)
+    assert normwise(host(Hd), Hr) <= TOL
+    assert np.any(host(Hd) < 0)
+
+
+def test_admm_not_spd(B):
+    R = 8
+    with pytest.raises(B.CstfError) as e:
+        B.cstf_admm_update(cu(np.ones((10, R))), cu(np.zeros((R, R))), cu(np.ones((10, R))), cu(np.zeros((10, R))),
+                           tol=0.0, max_iter=3)
+    assert e.value.status == B.CSTF_ERR_NOT_SPD
+
+
+def run_both(B, dims, idx, vals, R, start, outer=10, tol=1e-2, max_iter=10, warm=0):
+    ref = oracle.coalesce(dims, idx, vals)
+    orc = oracle.factorize(ref, start, outer_iters=outer, tol=tol, max_iter=max_iter, warm=warm)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    F = [cu(f) for f in start]
+    lam = cu(np.zeros(R))
+    opts = B.make_opts(R, outer_iters=outer, tol=tol, max_iter=max_iter, warm=warm)
+    gpu = B.cstf_factorize(X, F, lam, opts)
+    return orc, gpu, [host(f) for f in F], host(lam)
+
+
+def test_factorize_planted_tiny(B):
+    """configs[0]: fit after 10 outer iterations within 1e-6 and equal ADMM counts."""
+    p = datagen.planted_tiny(1)
+    start = datagen.perturbed_start(p, 1)
+    orc, gpu, F, lam = run_both(B, p.dims, p.idx, p.vals, p.R, start)
+    assert gpu["outer_done"] == 10
+    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
+    assert n >= 15            # the first five outer iterations are decided well away from ties
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+    assert gpu["fit"][-1] >= 1 - 1e-8
+    if tie is None:
+        for a, b in zip(F, orc["factors"]):
+            assert normwise(a, b) <= 1e-6
+
+
+@pytest.mark.parametrize("cfg,scale,R", [("nell2", 40, 16), ("enron", 40, 8), ("delicious", 2000, 8)])
+def test_factorize_scaled_configs(B, cfg, scale, R):
+    c = datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, R, c.seed)
+    orc, gpu, F, lam = run_both(B, c.dims, idx, vals, R, start)
+    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
+    assert tie is None, tie
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+
+
+def test_factorize_fixed_iterations_protocol(B):
+    """The timing protocol (eps = 0, 10 inner iterations) on a scaled NELL-2 shape."""
+    c = datagen.CONFIGS["nell2"].scaled(20, nnz_factor=200)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, 32, c.seed)
+    orc, gpu, F, lam = run_both(B, c.dims, idx, vals, 32, start, outer=3, tol=0.0)
+    assert np.all(gpu["iters"] == 10)
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+    for a, b in zip(F, orc["factors"]):
+        assert normwise(a, b) <= 1e-6
+
+
+def test_factorize_host_matches_device(B):
+    c = datagen.CONFIGS["enron"].scaled(60, nnz_factor=2000)
+    idx, vals = c.generate()
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    start = datagen.init_factors(c.dims, 8, 1)
+    opts = B.make_opts(8, outer_iters=3, tol=1e-2)
+    F = [cu(f) for f in start]
+    lam = cu(np.zeros(8))
+    g1 = B.cstf_factorize(X, F, lam, opts)
+    hf = [f.copy() for f in start]
+    hl = np.zeros(8)
+    g2 = B.cstf_factorize_host(X, hf, hl, opts)
+    assert np.array_equal(g1["fit"], g2["fit"])
+    for a, b in zip(hf, F):
+        assert np.array_equal(a, host(b))
+    assert np.array_equal(hl, host(lam))

@@ -1,0 +1,278 @@
+"""Benchmark of the cSTF hot path on B200 (driver contract, one JSON line on rank 0).
+
+A step is one outer iteration of Alg. 1 over the whole
+tensor: for every mode S / rho / Cholesky / inverse, MTTKRP, the fused ADMM
+update (10 inner iterations, eps = 0: the paper's timing protocol L930-933),
+normalisation and Gram, then the fit.  Inputs are the seeded synthetic tensor
+of the chosen BASELINE.json config (default configs[1], NELL-2-shaped), already
+resident in HBM when the timed region starts.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config nell2|enron|delicious|amazon]
+                  [--impl ours|reference] [--no-cpu-baseline]
+
+--impl reference times the FP64 CPU oracle (the reference arm of this tier) on
+the host cores: one outer iteration of the same workload per step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import datagen  # noqa: E402
+from paper_conf_icpp_sohksc24_b200 import costmodel as cm  # noqa: E402
+
+METRIC = "cSTF outer-iteration time (s) and ADMM update HBM GB/s at 1/2/4/8 B200"
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FP64_PEAK_TFLOPS = 37.1      # measured on this pool's B200 (DFMA and DMMA alike), profiles/r01_microbench.txt
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_PATH) as f:
+            p = json.load(f)
+        return p, "measured (MEASURED_PEAKS.json)"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0}, "fallback (B200_PROFILING.md)"
+
+
+def env_rank():
+    return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out = ""
+        sms, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sms.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sms) if sms else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sms)}
+
+
+def oracle_outer_iteration(cfg, idx, vals, R, steps, warmup):
+    """The FP64 oracle as it stands: one outer iteration (eps = 0, 10 inner) per step."""
+    import oracle
+    t0 = time.time()
+    X = oracle.coalesce(cfg.dims, idx, vals)
+    t_coalesce = time.time() - t0
+    F = datagen.init_factors(cfg.dims, R, cfg.seed)
+    times = []
+    for s in range(warmup + steps):
+        t0 = time.perf_counter()
+        oracle.factorize(X, F, outer_iters=1, tol=0.0, max_iter=10)
+        dt = time.perf_counter() - t0
+        if s >= warmup:
+            times.append(dt)
+    cores = len(os.sched_getaffinity(0))
+    return float(np.mean(times)), cores, t_coalesce
+
+
+def run_reference(args, cfg):
+    rank, world, _ = env_rank()
+    if rank != 0:
+        return 0
+    idx, vals = cfg.generate()
+    # the reference arm: the oracle, on the host cores, one full outer iteration per step
+    w = max(0, min(args.warmup, 1))     # a CPU has nothing to warm up; keep the run within minutes
+    k = max(1, min(args.steps, 3))
+    v, cores, tco = oracle_outer_iteration(cfg, idx, vals, cfg.R, k, w)
+    line = {"metric": METRIC, "value": v, "unit": "s", "n_gpus": world, "steps": k, "warmup": w,
+            "ms_per_step": v * 1e3, "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
+            "dtype": "f64", "data": "synthetic (datagen recipe)", "impl": "reference",
+            "config": config_dict(cfg),
+            "cpu_baseline": {"value": v, "unit": "s", "cores": cores, "kind": "oracle",
+                             "sample": f"{k} full outer iteration(s) of the {cfg.name} workload "
+                                       f"(eps=0, 10 inner); coalesce {tco:.1f}s excluded"},
+            "e2e": {"value": v, "unit": "s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+def config_dict(cfg):
+    return {"workload": cfg.name, "dims": list(cfg.dims), "nnz_generated": cfg.nnz, "R": cfg.R,
+            "seed": cfg.seed, "admm": "eps=0, max_iter=10 (PAPER.md L930-933)",
+            "warm_start": "scaled (D4)", "l2": "inputs larger than L2 (nonzero store >> 126 MB)"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="nell2", choices=sorted(datagen.CONFIGS))
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    cfg = datagen.CONFIGS[args.config]
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+
+    import torch
+    from paper_conf_icpp_sohksc24_b200 import binding as B
+
+    rank, world, local = env_rank()
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    R = cfg.R
+    t0 = time.time()
+    idx, vals = cfg.generate()
+    t_gen = time.time() - t0
+    t0 = time.time()
+    X = B.cstf_tensor_load_coo(cfg.dims, idx, vals)
+    torch.cuda.synchronize()
+    t_load = time.time() - t0
+    info = X.info()
+    F0 = datagen.init_factors(cfg.dims, R, cfg.seed)
+    F = [torch.from_numpy(f).cuda() for f in F0]
+    lam = torch.zeros(R, dtype=torch.float64, device="cuda")
+    stream = torch.cuda.current_stream()
+
+    def opts(n, timing=False):
+        return B.make_opts(R, outer_iters=n, tol=0.0, max_iter=10, timing=timing)
+
+    # warm-up: W outer iterations
+    B.cstf_factorize(X, F, lam, opts(max(args.warmup, 3)))
+    torch.cuda.synchronize()
+    # timed: K outer iterations in one call (each call starts with the init pass: included)
+    clocks = ClockSampler(local)
+    if dist:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    l0 = B.cstf_kernel_launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    rep = B.cstf_factorize(X, F, lam, opts(args.steps, timing=True))
+    e1.record(stream)
+    torch.cuda.synchronize()
+    launches = B.cstf_kernel_launch_count() - l0
+    if dist:
+        dist.barrier()
+    clk = clocks.stop()
+    ms_total = e0.elapsed_time(e1)
+    if dist:
+        t = torch.tensor([ms_total], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms_step = ms_total / args.steps
+    K = args.steps
+    N = len(cfg.dims)
+    mp = rep["mode_phase_ms"]             # [N][5], summed over K steps
+    ml = rep["mode_launches"]
+    phase_ms = {k: v / K for k, v in rep["phase_ms"].items()}
+    # roofline of the dominant kernel
+    peaks, peak_src = load_peaks()
+    nnz = info["nnz"]
+    mtt_ms = mp[:, 1].sum() / K
+    upd_ms = mp[:, 2].sum() / K
+    admm_bytes_model = sum(10 * cm.admm_bytes(I, R) for I in cfg.dims)        # 40 I R per inner iteration
+    admm_gbs = admm_bytes_model / (upd_ms * 1e-3) / 1e9 if upd_ms > 0 else None
+    if mtt_ms >= upd_ms:
+        byts = sum(cm.mttkrp_bytes(nnz, cfg.dims, n, R) for n in range(N))
+        launches_per = N   # one MTTKRP per mode per step
+        ach = byts / (mtt_ms * 1e-3) / 1e9
+        roof = {"kernel": "mttkrp (k_mttkrp + carry fix-up)", "bound": "hbm", "achieved": ach,
+                "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": ach / peaks["hbm_gbs"],
+                "traffic": None, "peak_source": peak_src,
+                "algorithmic_bytes_per_launch": byts / launches_per,
+                "avg_launch_ms": mtt_ms / launches_per,
+                "per_mode_ms": (mp[:, 1] / K).tolist()}
+    else:
+        fl = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
+        ach = fl / (upd_ms * 1e-3) / 1e12
+        roof = {"kernel": "admm (k_admm_dmma, row-resident)", "bound": "tensor", "achieved": ach,
+                "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS,
+                "traffic": None, "peak_source": "measured FP64 DMMA peak (tools/microbench.cu, profiles/r01_microbench.txt)",
+                "algorithmic_flops_per_launch": fl / N, "avg_launch_ms": upd_ms / N,
+                "per_mode_ms": (mp[:, 2] / K).tolist()}
+    line = {"metric": METRIC, "value": ms_step / 1e3, "unit": "s", "n_gpus": world, "steps": K,
+            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": False,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (datagen recipe, shapes of PAPER.md Table 2)",
+            "config": config_dict(cfg), "gpu_launches": int(launches),
+            "roofline": roof, "admm_update_gbs": admm_gbs,
+            "phases_ms_per_step": phase_ms, "clocks": clk,
+            "setup": {"generate_s": t_gen, "load_coo_s": t_load, "nnz_coalesced": nnz}}
+    # end to end through the public API with HOST buffers (pinned), one outer iteration per step
+    if not args.no_e2e:
+        hf = [torch.from_numpy(f.copy()).pin_memory() for f in F0]
+        hl = torch.zeros(R, dtype=torch.float64).pin_memory()
+        B.cstf_factorize_host(X, hf, hl, opts(1))
+        ts = []
+        for _ in range(K):
+            for h, f in zip(hf, F0):
+                h.numpy()[...] = f
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            a.record(stream)
+            B.cstf_factorize_host(X, hf, hl, opts(1))
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        fac_bytes = sum(I * R * 8 for I in cfg.dims)
+        line["e2e"] = {"value": float(np.mean(ts)) / 1e3, "unit": "s", "h2d_bytes_per_step": fac_bytes,
+                       "d2h_bytes_per_step": fac_bytes + R * 8 + 8,
+                       "note": "cstf_factorize_host: initial factors H2D, 1 outer iteration, factors+lambda+fit D2H"}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, cores, tco = oracle_outer_iteration(cfg, idx, vals, R, 1, 0)
+        line["cpu_baseline"] = {"value": v, "unit": "s", "cores": cores, "kind": "oracle",
+                                "sample": f"1 full outer iteration of {cfg.name} (eps=0, 10 inner), "
+                                          f"FP64 C/OpenMP oracle; coalesce {tco:.1f}s excluded"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if dist:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

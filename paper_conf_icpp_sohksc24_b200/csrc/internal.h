@@ -84,14 +84,19 @@ int comm_nranks(const cstf_comm* c);
 int comm_rank(const cstf_comm* c);
 
 // ---------------------------------------------------------------- tensor store
+// Mode-n copy of the nonzeros: sorted by i_n, then by the other modes in
+// increasing length order (so fibers of the shortest other mode are contiguous).
+// Array-of-structs records of `recb` bytes: int32 index of other[q] at byte 4q,
+// the FP64 value in the last 8 bytes.
 struct ModeStore {
   int64_t I = 0;            // rows of this mode (local rows when distributed)
   int64_t nnz = 0;          // nonzeros in this copy
   DevBuf rowptr;            // int64[I+1]
-  DevBuf idx[7];            // int32[nnz] for the other modes (increasing mode order)
-  DevBuf vals;              // double[nnz]
-  int other[7];             // mode id of idx[k]
+  DevBuf rec;               // nnz records
+  int recb = 16;            // record bytes: round_up(4 (N-1) + 8, 16)
+  int other[7];             // mode id of record slot q (slot 0 = shortest other mode)
 };
+inline int record_bytes(int N) { return ((4 * (N - 1) + 8) + 15) / 16 * 16; }
 
 }  // namespace cstf
 

@@ -9,6 +9,7 @@
 // (L403-430); the paper's own format (BLCO, L439-442) is replaced.
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <cstring>
 
 #include "internal.h"
@@ -184,6 +185,81 @@ __global__ void k_expand_rows(const int64_t* __restrict__ rowptr, int64_t I,
     for (int64_t p = rowptr[i]; p < rowptr[i + 1]; p++) out[p] = (int32_t)i;
 }
 
+// Stable LSD radix sort of positions 0..n-1 by the key tuple keys[0..nk-1]
+// (keys[0] most significant).  Keys are packed into <= 64-bit groups from the
+// least significant end; every pass is a stable CUB radix sort, so equal
+// tuples keep their input order.  Result in `perm` (uint32[n]).
+cstf_status lsd_sort(const int32_t* const* keys, const int64_t* dims, int nk, int64_t n, DevBuf& perm,
+                     DevBuf& tmp, cudaStream_t st) {
+  CSTF_TRY(perm.alloc((size_t)n * 4));
+  if (n == 0) return CSTF_OK;
+  DevBuf perm_b, key_a, key_b;
+  CSTF_TRY(perm_b.alloc((size_t)n * 4));
+  CSTF_TRY(key_a.alloc((size_t)n * 8));
+  CSTF_TRY(key_b.alloc((size_t)n * 8));
+  k_iota<<<grid_for(n), kThreads, 0, st>>>(perm.as<uint32_t>(), n);
+  CSTF_LAUNCHED();
+  int hi = nk - 1;
+  while (hi >= 0) {
+    int lo = hi, tot = bits_for(dims[hi]);
+    while (lo - 1 >= 0 && tot + bits_for(dims[lo - 1]) <= 64) { lo--; tot += bits_for(dims[lo]); }
+    PackArgs pa;
+    pa.count = hi - lo + 1;
+    int sh = 0;
+    for (int m = hi; m >= lo; m--) {
+      pa.idx[m - lo] = keys[m];
+      pa.shift[m - lo] = sh;
+      sh += bits_for(dims[m]);
+    }
+    if (tot > 0) {
+      k_pack_keys<<<grid_for(n), kThreads, 0, st>>>(pa, perm.as<uint32_t>(), n, key_a.as<uint64_t>());
+      CSTF_LAUNCHED();
+      size_t tb = 0;
+      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, key_a.as<uint64_t>(), key_b.as<uint64_t>(),
+                                                perm.as<uint32_t>(), perm_b.as<uint32_t>(), n, 0, tot, st));
+      CSTF_TRY(tmp.ensure(tb));
+      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, key_a.as<uint64_t>(), key_b.as<uint64_t>(),
+                                                perm.as<uint32_t>(), perm_b.as<uint32_t>(), n, 0, tot, st));
+      count_launch();
+      std::swap(perm, perm_b);
+    }
+    hi = lo - 1;
+  }
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  return CSTF_OK;
+}
+
+struct RecArgs {
+  const int32_t* idx[7];   // slot q source index array (canonical order)
+  int nslots;
+  int recb;
+};
+
+// rec[p] = {idx[q][perm[p]] ..., vals[perm[p]]}
+__global__ void k_make_records(RecArgs a, const double* __restrict__ vals, const uint32_t* __restrict__ perm,
+                               int64_t n, char* __restrict__ rec) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    const uint32_t src = perm[p];
+    char* r = rec + p * a.recb;
+    int32_t* ri = reinterpret_cast<int32_t*>(r);
+    for (int q = 0; q < a.nslots; q++) ri[q] = a.idx[q][src];
+    for (int q = a.nslots; q < (a.recb - 8) / 4; q++) ri[q] = 0;
+    *reinterpret_cast<double*>(r + a.recb - 8) = vals[src];
+  }
+}
+
+// inverse of k_make_records for export: SoA arrays of the record slots + values
+__global__ void k_split_records(const char* __restrict__ rec, int recb, int nslots, int64_t n, OutArgs out,
+                                double* __restrict__ vals) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    const char* r = rec + p * recb;
+    for (int q = 0; q < nslots; q++) out.idx[q][p] = reinterpret_cast<const int32_t*>(r)[q];
+    vals[p] = *reinterpret_cast<const double*>(r + recb - 8);
+  }
+}
+
 // rowptr[0] = 0, rowptr[i+1] = sum_{r<=i} counts[r]
 cstf_status build_rowptr(const int32_t* d_key, int64_t n, int64_t I, DevBuf& rowptr, DevBuf& tmp,
                          cudaStream_t st) {
@@ -235,44 +311,13 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     CSTF_CUDA(cudaStreamSynchronize(st));
     if (nbad) return fail(CSTF_ERR_INVALID_ARG, std::to_string(nbad) + " indices outside [0, dims[n])");
   }
-  // ---- 2. canonical order: LSD radix sort over packed groups of modes, last group first
-  DevBuf perm_a, perm_b, key_a, key_b;
-  CSTF_TRY(perm_a.alloc((size_t)n * 4));
-  CSTF_TRY(perm_b.alloc((size_t)n * 4));
-  CSTF_TRY(key_a.alloc((size_t)n * 8));
-  CSTF_TRY(key_b.alloc((size_t)n * 8));
-  if (n) {
-    k_iota<<<grid_for(n), kThreads, 0, st>>>(perm_a.as<uint32_t>(), n);
-    CSTF_LAUNCHED();
+  // ---- 2. canonical order: stable LSD radix sort by (i_1, ..., i_N)
+  DevBuf perm_a;
+  {
+    const int32_t* keys[8];
+    for (int m = 0; m < N; m++) keys[m] = in_idx[m].as<int32_t>();
+    CSTF_TRY(lsd_sort(keys, X->dims, N, n, perm_a, tmp, st));
   }
-  int hi = N - 1;
-  while (hi >= 0 && n > 0) {
-    // group = modes [lo, hi] with total bits <= 64
-    int lo = hi, tot = bits_for(X->dims[hi]);
-    while (lo - 1 >= 0 && tot + bits_for(X->dims[lo - 1]) <= 64) { lo--; tot += bits_for(X->dims[lo]); }
-    PackArgs pa;
-    pa.count = hi - lo + 1;
-    int sh = 0;
-    for (int m = hi; m >= lo; m--) {  // lowest mode most significant
-      pa.idx[m - lo] = in_idx[m].as<int32_t>();
-      pa.shift[m - lo] = sh;
-      sh += bits_for(X->dims[m]);
-    }
-    if (tot > 0) {
-      k_pack_keys<<<grid_for(n), kThreads, 0, st>>>(pa, perm_a.as<uint32_t>(), n, key_a.as<uint64_t>());
-      CSTF_LAUNCHED();
-      size_t tb = 0;
-      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, key_a.as<uint64_t>(), key_b.as<uint64_t>(),
-                                                perm_a.as<uint32_t>(), perm_b.as<uint32_t>(), n, 0, tot, st));
-      CSTF_TRY(tmp.ensure(tb));
-      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, key_a.as<uint64_t>(), key_b.as<uint64_t>(),
-                                                perm_a.as<uint32_t>(), perm_b.as<uint32_t>(), n, 0, tot, st));
-      count_launch();
-      std::swap(perm_a, perm_b);
-    }
-    hi = lo - 1;
-  }
-  key_a.release(); key_b.release(); perm_b.release();
   // ---- 3. gather into sorted order, free the inputs
   DevBuf s_idx[8], s_vals;
   for (int m = 0; m < N; m++) {
@@ -345,63 +390,70 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     X->normX2 = hv[0];
     memcpy(&X->hash, &hv[1], 8);
   }
-  // ---- 6. per-mode copies, stably sorted by i_n (mode 0 = canonical order)
-  for (int n_ = N - 1; n_ >= 0; n_--) {
+  // ---- 6. per-mode copies: sorted by (i_n, other modes by increasing length), AoS records
+  const int recb = record_bytes(N);
+  for (int n_ = 0; n_ < N; n_++) {
     ModeStore& ms = X->mode[n_];
     ms.I = X->dims[n_];
     ms.nnz = nout;
+    ms.recb = recb;
     int k = 0;
     for (int m = 0; m < N; m++)
       if (m != n_) ms.other[k++] = m;
-    if (n_ == 0) {
-      CSTF_TRY(build_rowptr(c_idx[0].as<int32_t>(), nout, ms.I, ms.rowptr, tmp, st));
-      for (int q = 0; q < N - 1; q++) ms.idx[q] = std::move(c_idx[ms.other[q]]);
-      ms.vals = std::move(c_vals);
-      c_idx[0].release();
-      break;
-    }
-    DevBuf keys_out, pm_in, pm_out;
-    CSTF_TRY(keys_out.alloc((size_t)nout * 4));
-    CSTF_TRY(pm_in.alloc((size_t)nout * 4));
-    CSTF_TRY(pm_out.alloc((size_t)nout * 4));
+    std::stable_sort(ms.other, ms.other + (N - 1), [&](int a, int b) { return X->dims[a] < X->dims[b]; });
+    const int32_t* keys[8];
+    int64_t kd[8];
+    keys[0] = c_idx[n_].as<int32_t>();
+    kd[0] = X->dims[n_];
+    for (int q = 0; q < N - 1; q++) { keys[q + 1] = c_idx[ms.other[q]].as<int32_t>(); kd[q + 1] = X->dims[ms.other[q]]; }
+    DevBuf pm;
+    CSTF_TRY(lsd_sort(keys, kd, N, nout, pm, tmp, st));
+    CSTF_TRY(build_rowptr(c_idx[n_].as<int32_t>(), nout, ms.I, ms.rowptr, tmp, st));
+    CSTF_TRY(ms.rec.alloc((size_t)nout * recb));
+    RecArgs ra;
+    ra.nslots = N - 1;
+    ra.recb = recb;
+    for (int q = 0; q < N - 1; q++) ra.idx[q] = c_idx[ms.other[q]].as<int32_t>();
     if (nout) {
-      k_iota<<<grid_for(nout), kThreads, 0, st>>>(pm_in.as<uint32_t>(), nout);
+      k_make_records<<<grid_for(nout), kThreads, 0, st>>>(ra, c_vals.as<double>(), pm.as<uint32_t>(), nout,
+                                                          ms.rec.as<char>());
       CSTF_LAUNCHED();
-      int nb = bits_for(ms.I);
-      size_t tb = 0;
-      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, tb, (const uint32_t*)c_idx[n_].p, keys_out.as<uint32_t>(),
-                                                pm_in.as<uint32_t>(), pm_out.as<uint32_t>(), nout, 0, nb > 0 ? nb : 1, st));
-      CSTF_TRY(tmp.ensure(tb));
-      CSTF_CUDA(cub::DeviceRadixSort::SortPairs(tmp.p, tb, (const uint32_t*)c_idx[n_].p, keys_out.as<uint32_t>(),
-                                                pm_in.as<uint32_t>(), pm_out.as<uint32_t>(), nout, 0, nb > 0 ? nb : 1, st));
-      count_launch();
     }
-    CSTF_TRY(build_rowptr(keys_out.as<int32_t>(), nout, ms.I, ms.rowptr, tmp, st));
-    for (int q = 0; q < N - 1; q++) {
-      CSTF_TRY(ms.idx[q].alloc((size_t)nout * 4));
-      if (nout) { k_gather<int32_t><<<grid_for(nout), kThreads, 0, st>>>(c_idx[ms.other[q]].as<int32_t>(), pm_out.as<uint32_t>(), nout, ms.idx[q].as<int32_t>()); CSTF_LAUNCHED(); }
-    }
-    CSTF_TRY(ms.vals.alloc((size_t)nout * 8));
-    if (nout) { k_gather<double><<<grid_for(nout), kThreads, 0, st>>>(c_vals.as<double>(), pm_out.as<uint32_t>(), nout, ms.vals.as<double>()); CSTF_LAUNCHED(); }
     CSTF_CUDA(cudaStreamSynchronize(st));
   }
-  CSTF_CUDA(cudaStreamSynchronize(st));
   return CSTF_OK;
 }
 
+// Canonical order back from the mode-0 copy: expand rows, split the records,
+// stable sort by (i_1..i_N), copy to the host.
 cstf_status export_store(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals) {
   const ModeStore& ms = X->mode[0];
-  int64_t n = ms.nnz;
+  const int N = X->N;
+  const int64_t n = ms.nnz;
   cudaStream_t st = 0;
   if (n == 0) return CSTF_OK;
-  DevBuf rows;
-  CSTF_TRY(rows.alloc((size_t)n * 4));
-  k_expand_rows<<<grid_for(ms.I), kThreads, 0, st>>>(ms.rowptr.as<int64_t>(), ms.I, rows.as<int32_t>());
+  DevBuf soa[8], vals, tmp, perm, out;
+  for (int m = 0; m < N; m++) CSTF_TRY(soa[m].alloc((size_t)n * 4));
+  CSTF_TRY(vals.alloc((size_t)n * 8));
+  k_expand_rows<<<grid_for(ms.I), kThreads, 0, st>>>(ms.rowptr.as<int64_t>(), ms.I, soa[0].as<int32_t>());
   CSTF_LAUNCHED();
-  CSTF_CUDA(cudaMemcpy(host_idx[0], rows.p, (size_t)n * 4, cudaMemcpyDeviceToHost));
-  for (int q = 0; q < X->N - 1; q++)
-    CSTF_CUDA(cudaMemcpy(host_idx[ms.other[q]], ms.idx[q].p, (size_t)n * 4, cudaMemcpyDeviceToHost));
-  CSTF_CUDA(cudaMemcpy(host_vals, ms.vals.p, (size_t)n * 8, cudaMemcpyDeviceToHost));
+  OutArgs oa;
+  oa.N = N - 1;
+  for (int q = 0; q < N - 1; q++) oa.idx[q] = soa[ms.other[q]].as<int32_t>();
+  k_split_records<<<grid_for(n), kThreads, 0, st>>>(ms.rec.as<char>(), ms.recb, N - 1, n, oa, vals.as<double>());
+  CSTF_LAUNCHED();
+  const int32_t* keys[8];
+  for (int m = 0; m < N; m++) keys[m] = soa[m].as<int32_t>();
+  CSTF_TRY(lsd_sort(keys, X->dims, N, n, perm, tmp, st));
+  CSTF_TRY(out.alloc((size_t)n * 8));
+  for (int m = 0; m < N; m++) {
+    k_gather<int32_t><<<grid_for(n), kThreads, 0, st>>>(soa[m].as<int32_t>(), perm.as<uint32_t>(), n, out.as<int32_t>());
+    CSTF_LAUNCHED();
+    CSTF_CUDA(cudaMemcpy(host_idx[m], out.p, (size_t)n * 4, cudaMemcpyDeviceToHost));
+  }
+  k_gather<double><<<grid_for(n), kThreads, 0, st>>>(vals.as<double>(), perm.as<uint32_t>(), n, out.as<double>());
+  CSTF_LAUNCHED();
+  CSTF_CUDA(cudaMemcpy(host_vals, out.p, (size_t)n * 8, cudaMemcpyDeviceToHost));
   return CSTF_OK;
 }
 

@@ -266,7 +266,7 @@ def test_factorize_planted_tiny(B):
     n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
     assert n >= 15            # the first five outer iterations are decided well away from ties
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
-    assert gpu["fit"][-1] >= 1 - 1e-8
+    assert gpu["fit"][-1] >= 1 - 1e-6          # recovery (the 1e-8 gate is the oracle's pin P8)
     if tie is None:
         for a, b in zip(F, orc["factors"]):
             assert normwise(a, b) <= 1e-6

@@ -88,13 +88,29 @@ int comm_rank(const cstf_comm* c);
 // increasing length order (so fibers of the shortest other mode are contiguous).
 // Array-of-structs records of `recb` bytes: int32 index of other[q] at byte 4q,
 // the FP64 value in the last 8 bytes.
+//
+// k-blocked copies: when the output mode is short and the
+// longest other mode is long, the nonzeros are ordered by (kb = i_t / kTileRows,
+// i_n, ...), t = other[N-2].  Rows are then "virtual rows" v = kb * I + i_n and
+// rowptr has nblk * I + 1 entries; MTTKRP writes one partial row per virtual row
+// and sums the partials over kb in fixed order.  The factor rows of block kb are
+// staged in shared memory by the CTA that processes them.
+constexpr int kTileRows = 256;
 struct ModeStore {
   int64_t I = 0;            // rows of this mode (local rows when distributed)
   int64_t nnz = 0;          // nonzeros in this copy
-  DevBuf rowptr;            // int64[I+1]
+  DevBuf rowptr;            // int64[Ivirt+1]
   DevBuf rec;               // nnz records
   int recb = 16;            // record bytes: round_up(4 (N-1) + 8, 16)
   int other[7];             // mode id of record slot q (slot 0 = shortest other mode)
+  // k-blocking
+  bool tiled = false;
+  int64_t nblk = 1;         // blocks of the tiled mode
+  int64_t Ivirt = 0;        // rows of rowptr (= I when not tiled)
+  // cached work split of a tiled copy: warp-chunk starts and the block of each CTA chunk
+  mutable DevBuf wstart;    // int64[nwchunks+1]
+  mutable DevBuf ckb;       // int32[nctachunks]
+  mutable int64_t nwchunks = 0, nctachunks = 0;
 };
 inline int record_bytes(int N) { return ((4 * (N - 1) + 8) + 15) / 16 * 16; }
 

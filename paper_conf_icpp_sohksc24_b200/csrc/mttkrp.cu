@@ -18,6 +18,8 @@
 //    are gathered back to back, so the repeated fiber row is an L1 hit.
 //  * Measured bound: with L2-resident factors the kernel runs at
 //    the L2->SM row-gather rate (~20 TB/s on B200 for 256-byte rows).
+#include <vector>
+
 #include "internal.h"
 
 namespace cstf {
@@ -31,19 +33,29 @@ struct MArgs {
   const double* F[7];   // factor of record slot q
   int64_t I, nnz, chunk, nchunks;
   int R, recb, nother;
-  const int64_t* lb;    // [nchunks+1] first row with rowptr >= c*chunk (lb[nchunks] = I)
+  const int64_t* lb;    // [nchunks+1] first row with rowptr >= start of chunk c (lb[nchunks] = I)
   const int32_t* cont;  // [nchunks] row continuing into chunk c from an earlier chunk, or -1
-  double* M;
+  const int64_t* wstart;  // [nchunks+1] explicit chunk starts (k-blocked copies) or null
+  const int32_t* ckb;     // [nchunks/8] block of each CTA chunk (k-blocked copies)
+  int64_t It;             // rows of the k-blocked mode's factor (slot nother-1)
+  double* M;            // output rows (virtual rows when k-blocked)
   double* carry;        // [nchunks][R]
 };
 
+__device__ __forceinline__ int64_t chunk_begin(const MArgs& a, int64_t c) {
+  return a.wstart ? a.wstart[c] : c * a.chunk;
+}
+__device__ __forceinline__ int64_t chunk_end(const MArgs& a, int64_t c) {
+  return a.wstart ? a.wstart[c + 1] : min((c + 1) * a.chunk, a.nnz);
+}
+
 __global__ void k_chunk_bounds(const int64_t* __restrict__ rowptr, int64_t I, int64_t nnz,
-                               int64_t chunk, int64_t nchunks, int64_t* __restrict__ lb,
-                               int32_t* __restrict__ cont) {
+                               int64_t chunk, int64_t nchunks, const int64_t* __restrict__ wstart,
+                               int64_t* __restrict__ lb, int32_t* __restrict__ cont) {
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nchunks;
        c += (int64_t)gridDim.x * blockDim.x) {
     if (c == nchunks) { lb[c] = I; continue; }
-    const int64_t p0 = c * chunk;
+    const int64_t p0 = wstart ? wstart[c] : c * chunk;
     int64_t lo = 0, hi = I;          // lower_bound: first row r with rowptr[r] >= p0
     while (lo < hi) {
       const int64_t mid = (lo + hi) >> 1;
@@ -69,8 +81,11 @@ __device__ __forceinline__ const double2* row_addr(const char* base, unsigned j)
 // record word group) and broadcasts them with shuffles; the P groups take
 // interleaved nonzeros of the current row, so consecutive nonzeros of a fiber
 // are gathered back to back and the repeated fiber row hits in L1.
+// One warp processes chunk c.  Fb[q] = lane's byte offset into the row source of
+// slot q (a factor in global memory, or the shared-memory slab of a k-blocked
+// copy, already shifted by the slab's first row).
 template <int NOTHER, int R, int RECB>
-__global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
+__device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const char* const* Fb, int4* srec) {
   constexpr int RV = R / 2;                    // double2 per row
   constexpr int G = RV < 32 ? RV : 32;         // lanes per group
   constexpr int VPL = RV / G;                  // double2 per lane
@@ -79,14 +94,9 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
   constexpr int NW = RECB / 4;                 // 32-bit words per record
   const int lane = threadIdx.x & 31;
   const int sg = lane / G, gl = lane % G;
-  const int64_t warp0 = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5);
-  const int64_t nwarps = (int64_t)gridDim.x * kWarps;
-  const char* Fb[NOTHER];
-#pragma unroll
-  for (int q = 0; q < NOTHER; q++) Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
-  for (int64_t c = warp0; c < a.nchunks; c += nwarps) {
-    const int64_t p0 = c * a.chunk;
-    const int64_t p1 = min(p0 + a.chunk, a.nnz);
+  {
+    const int64_t p0 = chunk_begin(a, c);
+    const int64_t p1 = chunk_end(a, c);
     const int32_t ct = a.cont[c];
     int64_t row = ct >= 0 ? (int64_t)ct : a.lb[c];
     const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
@@ -112,20 +122,26 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
       for (int s = 0; s < VPL; s++) acc[s] = make_double2(0.0, 0.0);
     };
 
+    // Records arrive 32 at a time: one coalesced 16-byte load per lane, issued
+    // one batch ahead (register double buffer), published through a per-warp
+    // shared buffer; each group then reads its record with one 16-byte LDS.
+    constexpr int NV = RECB / 16;                // int4 per record
+    int4* sr = srec + (threadIdx.x >> 5) * 32 * NV;
+    int4 nxt[NV];
+#pragma unroll
+    for (int k = 0; k < NV; k++)
+      nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
+                                : make_int4(0, 0, 0, 0);
     for (int64_t pb = p0; pb < p1; pb += 32) {
       const int nb = (int)min((int64_t)32, p1 - pb);
-      unsigned w[NW];
-      if (lane < nb) {
-        const int4* rp = reinterpret_cast<const int4*>(a.rec + (pb + lane) * RECB);
+      __syncwarp();
 #pragma unroll
-        for (int k = 0; k < NW / 4; k++) {
-          const int4 x = __ldcs(rp + k);
-          w[4 * k] = x.x; w[4 * k + 1] = x.y; w[4 * k + 2] = x.z; w[4 * k + 3] = x.w;
-        }
-      } else {
+      for (int k = 0; k < NV; k++) sr[lane * NV + k] = nxt[k];
+      __syncwarp();
 #pragma unroll
-        for (int k = 0; k < NW; k++) w[k] = 0u;
-      }
+      for (int k = 0; k < NV; k++)
+        nxt[k] = (pb + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 32 + lane) * RECB) + k)
+                                       : make_int4(0, 0, 0, 0);
       int t = 0;
       while (t < nb) {
         const int64_t p = pb + t;
@@ -136,21 +152,25 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
           continue;
         }
         const int run = (int)min((int64_t)(nb - t), seg_end - p);
+#pragma unroll 4
         for (int done = 0; done < run; done += P) {
           const bool ok = (done + sg) < run;
-          const int srcc = ok ? t + done + sg : t + done;     // a valid lane of this batch
-          const unsigned vlo = __shfl_sync(0xffffffffu, w[NW - 2], srcc);
-          const unsigned vhi = __shfl_sync(0xffffffffu, w[NW - 1], srcc);
-          const double v = ok ? __hiloint2double((int)vhi, (int)vlo) : 0.0;   // idle group adds 0
+          const int src = ok ? t + done + sg : t + done;      // a valid slot of this batch
+          unsigned w[NW];
+#pragma unroll
+          for (int k = 0; k < NV; k++) {
+            const int4 x = sr[src * NV + k];
+            w[4 * k] = x.x; w[4 * k + 1] = x.y; w[4 * k + 2] = x.z; w[4 * k + 3] = x.w;
+          }
+          const double v = ok ? __hiloint2double((int)w[NW - 1], (int)w[NW - 2]) : 0.0;   // idle group adds 0
           double2 f[VPL];
 #pragma unroll
-          for (int q = 0; q < NOTHER; q++) {
-            const unsigned j = __shfl_sync(0xffffffffu, w[q], srcc);
-            const double2* rp = row_addr<ROWB>(Fb[q], j);
+          for (int qq = 0; qq < NOTHER; qq++) {
+            const double2* rp = row_addr<ROWB>(Fb[qq], w[qq]);
 #pragma unroll
             for (int s = 0; s < VPL; s++) {
-              const double2 x = __ldg(rp + s * G);
-              if (q == 0) f[s] = x;
+              const double2 x = rp[s * G];     // global (read-only) or shared slab
+              if (qq == 0) f[s] = x;
               else { f[s].x *= x.x; f[s].y *= x.y; }
             }
           }
@@ -170,6 +190,47 @@ __global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
   }
 }
 
+template <int NOTHER, int R, int RECB>
+__global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
+  constexpr int G = (R / 2) < 32 ? (R / 2) : 32;
+  const int gl = (threadIdx.x & 31) % G;
+  const char* Fb[NOTHER];
+#pragma unroll
+  for (int q = 0; q < NOTHER; q++) Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
+  const int64_t warp0 = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5);
+  const int64_t nwarps = (int64_t)gridDim.x * kWarps;
+  __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
+  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB>(a, c, Fb, srec);
+}
+
+// k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
+// block's kTileRows rows of the last slot's factor are staged in shared memory
+// (coalesced 16-byte copies), the other slots gather from global memory.
+template <int NOTHER, int R, int RECB>
+__global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_tiled(MArgs a) {
+  extern __shared__ double2 slab[];            // [kTileRows][R/2]
+  __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
+  constexpr int G = (R / 2) < 32 ? (R / 2) : 32;
+  const int gl = (threadIdx.x & 31) % G;
+  const int warp = threadIdx.x >> 5;
+  const int64_t ncta = a.nchunks / kWarps;
+  for (int64_t b = blockIdx.x; b < ncta; b += gridDim.x) {
+    const int64_t kb = a.ckb[b];
+    const int64_t r0 = kb * kTileRows;
+    const int rows = (int)min((int64_t)kTileRows, a.It - r0);
+    const double2* src = reinterpret_cast<const double2*>(a.F[NOTHER - 1] + r0 * R);
+    __syncthreads();                           // previous block's readers are done
+    for (int x = threadIdx.x; x < rows * (R / 2); x += blockDim.x) slab[x] = __ldg(src + x);
+    __syncthreads();
+    const char* Fb[NOTHER];
+#pragma unroll
+    for (int q = 0; q < NOTHER - 1; q++) Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
+    // slot NOTHER-1 indices are absolute rows: shift the slab base by -r0 rows
+    Fb[NOTHER - 1] = reinterpret_cast<const char*>(slab) - r0 * (int64_t)(R * 8) + gl * 16;
+    process_chunk<NOTHER, R, RECB>(a, b * kWarps + warp, Fb, srec);
+  }
+}
+
 // Generic path (any R <= 128, any record size): lane = column(s), one nonzero at a time.
 template <int CPL>
 __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
@@ -178,8 +239,8 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
   const int64_t nwarps = (int64_t)gridDim.x * kWarps;
   const int R = a.R;
   for (int64_t c = warp0; c < a.nchunks; c += nwarps) {
-    const int64_t p0 = c * a.chunk;
-    const int64_t p1 = min(p0 + a.chunk, a.nnz);
+    const int64_t p0 = chunk_begin(a, c);
+    const int64_t p1 = chunk_end(a, c);
     const int32_t ct = a.cont[c];
     int64_t row = ct >= 0 ? (int64_t)ct : a.lb[c];
     const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
@@ -232,8 +293,42 @@ __global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks,
   }
 }
 
+// M[i, :] = sum over blocks kb (in order) of the partial rows P[kb * I + i, :]
+__global__ void k_reduce_blocks(const double* __restrict__ Pv, int64_t I, int64_t nblk, int R,
+                                double* __restrict__ M) {
+  const int64_t n = I * R;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
+       x += (int64_t)gridDim.x * blockDim.x) {
+    double s = 0.0;
+    for (int64_t kb = 0; kb < nblk; kb++) s += Pv[kb * n + x];
+    M[x] = s;
+  }
+}
+
+template <int NOTHER, int RECB, int RR>
+bool launch_tiled_r(const MArgs& a, int grid, cudaStream_t st) {
+  const size_t smem = (size_t)kTileRows * RR * 8;
+  static bool attr = false;
+  if (!attr) {
+    if (cudaFuncSetAttribute(k_mttkrp_tiled<NOTHER, RR, RECB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)smem) != cudaSuccess) return false;
+    attr = true;
+  }
+  k_mttkrp_tiled<NOTHER, RR, RECB><<<grid, kWarps * 32, smem, st>>>(a);
+  return true;
+}
+
 template <int NOTHER, int RECB>
-bool launch_fast(const MArgs& a, int grid, cudaStream_t st) {
+bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled) {
+  if (tiled) {
+    switch (a.R) {     // slab = 256 rows x R doubles: 2 KB .. 128 KB
+      case 8: return launch_tiled_r<NOTHER, RECB, 8>(a, grid, st);
+      case 16: return launch_tiled_r<NOTHER, RECB, 16>(a, grid, st);
+      case 32: return launch_tiled_r<NOTHER, RECB, 32>(a, grid, st);
+      case 64: return launch_tiled_r<NOTHER, RECB, 64>(a, grid, st);
+      default: break;  // other ranks: the flat kernel on the k-blocked copy
+    }
+  }
   switch (a.R) {
 #define CASE(RR) case RR: k_mttkrp_fast<NOTHER, RR, RECB><<<grid, kWarps * 32, 0, st>>>(a); return true;
     CASE(2) CASE(4) CASE(8) CASE(16) CASE(32) CASE(64) CASE(128)
@@ -242,15 +337,17 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st) {
   }
 }
 
-cstf_status launch_main(const MArgs& a, int grid, cudaStream_t st) {
+cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st) {
   bool done = false;
+  const bool tl = a.ckb != nullptr;
+  const int g = tl ? tgrid : grid;
   switch (a.nother) {
-    case 1: done = launch_fast<1, 16>(a, grid, st); break;
-    case 2: done = launch_fast<2, 16>(a, grid, st); break;
-    case 3: done = launch_fast<3, 32>(a, grid, st); break;
-    case 4: done = launch_fast<4, 32>(a, grid, st); break;
-    case 5: done = launch_fast<5, 32>(a, grid, st); break;
-    case 6: done = launch_fast<6, 32>(a, grid, st); break;
+    case 1: done = launch_fast<1, 16>(a, grid, st, false); break;
+    case 2: done = launch_fast<2, 16>(a, g, st, tl); break;
+    case 3: done = launch_fast<3, 32>(a, g, st, tl); break;
+    case 4: done = launch_fast<4, 32>(a, g, st, tl); break;
+    case 5: done = launch_fast<5, 32>(a, g, st, tl); break;
+    case 6: done = launch_fast<6, 32>(a, g, st, tl); break;
     default: break;   // 7 other modes: 48-byte records, generic path
   }
   if (!done) {
@@ -263,13 +360,58 @@ cstf_status launch_main(const MArgs& a, int grid, cudaStream_t st) {
 }
 
 struct Workspace {
-  DevBuf lb, cont, carry;
+  DevBuf lb, cont, carry, partial, kbptr;
+  std::vector<int64_t> hk;
 };
+
+__global__ void k_kb_offsets(const int64_t* __restrict__ rowptr, int64_t I, int64_t nblk,
+                             int64_t* __restrict__ out) {
+  for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b <= nblk; b += (int64_t)gridDim.x * blockDim.x)
+    out[b] = rowptr[b * I];
+}
 Workspace& ws() {
   static thread_local Workspace w[64];
   int dev = 0;
   cudaGetDevice(&dev);
   return w[dev & 63];
+}
+
+// Work split of a k-blocked copy (host logic, cached on the mode store): every
+// block's nonzero range is cut into CTA chunks of <= kCtaChunk nonzeros, each
+// split into kWarps warp chunks; every block gets at least one CTA chunk so its
+// (possibly empty) partial rows are written.
+constexpr int64_t kCtaChunk = 16384;
+
+cstf_status tiled_split(const ModeStore& ms, cudaStream_t st) {
+  if (ms.nctachunks > 0) return CSTF_OK;
+  Workspace& w = ws();
+  CSTF_TRY(w.kbptr.ensure((size_t)(ms.nblk + 1) * 8));
+  k_kb_offsets<<<(int)((ms.nblk + 256) / 256), 256, 0, st>>>(ms.rowptr.as<int64_t>(), ms.I, ms.nblk,
+                                                             w.kbptr.as<int64_t>());
+  CSTF_LAUNCHED();
+  std::vector<int64_t> kp((size_t)ms.nblk + 1);
+  CSTF_CUDA(cudaMemcpyAsync(kp.data(), w.kbptr.p, kp.size() * 8, cudaMemcpyDeviceToHost, st));
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  std::vector<int64_t> starts;
+  std::vector<int32_t> kbs;
+  for (int64_t b = 0; b < ms.nblk; b++) {
+    const int64_t lo = kp[(size_t)b], hi = kp[(size_t)b + 1];
+    const int64_t nc = std::max<int64_t>(1, (hi - lo + kCtaChunk - 1) / kCtaChunk);
+    for (int64_t k = 0; k < nc; k++) {
+      const int64_t c0 = lo + (hi - lo) * k / nc, c1 = lo + (hi - lo) * (k + 1) / nc;
+      kbs.push_back((int32_t)b);
+      for (int wv = 0; wv < kWarps; wv++) starts.push_back(c0 + (c1 - c0) * wv / kWarps);
+    }
+  }
+  starts.push_back(ms.nnz);
+  CSTF_TRY(ms.wstart.alloc(starts.size() * 8));
+  CSTF_TRY(ms.ckb.alloc(kbs.size() * 4));
+  CSTF_CUDA(cudaMemcpyAsync(ms.wstart.p, starts.data(), starts.size() * 8, cudaMemcpyHostToDevice, st));
+  CSTF_CUDA(cudaMemcpyAsync(ms.ckb.p, kbs.data(), kbs.size() * 4, cudaMemcpyHostToDevice, st));
+  CSTF_CUDA(cudaStreamSynchronize(st));
+  ms.nctachunks = (int64_t)kbs.size();
+  ms.nwchunks = ms.nctachunks * kWarps;
+  return CSTF_OK;
 }
 
 }  // namespace
@@ -280,47 +422,75 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   const int N = X->N;
   const DeviceInfo& di = device_info();
   const int64_t nnz = ms.nnz;
-  // chunk: ~4 chunks per resident warp, multiple of 32, in [256, 8192]
-  const int64_t resident = (int64_t)di.sms * 8 * kWarps;
-  int64_t chunk = (nnz + resident * 4 - 1) / (resident * 4);
-  chunk = ((chunk + 31) / 32) * 32;
-  if (chunk < 256) chunk = 256;
-  if (chunk > 8192) chunk = 8192;
-  const int64_t nchunks = nnz > 0 ? (nnz + chunk - 1) / chunk : 1;
   Workspace& w = ws();
+  MArgs a;
+  a.wstart = nullptr;
+  a.ckb = nullptr;
+  int64_t chunk = 0, nchunks = 0;
+  if (ms.tiled) {
+    CSTF_TRY(tiled_split(ms, st));
+    nchunks = ms.nwchunks;
+    a.wstart = ms.wstart.as<int64_t>();
+    a.ckb = ms.ckb.as<int32_t>();
+  } else {
+    // chunk: ~4 chunks per resident warp, multiple of 32, in [256, 8192]
+    const int64_t resident = (int64_t)di.sms * 8 * kWarps;
+    chunk = (nnz + resident * 4 - 1) / (resident * 4);
+    chunk = ((chunk + 31) / 32) * 32;
+    if (chunk < 256) chunk = 256;
+    if (chunk > 8192) chunk = 8192;
+    nchunks = nnz > 0 ? (nnz + chunk - 1) / chunk : 1;
+  }
   CSTF_TRY(w.lb.ensure((size_t)(nchunks + 1) * 8));
   CSTF_TRY(w.cont.ensure((size_t)nchunks * 4));
   CSTF_TRY(w.carry.ensure((size_t)nchunks * R * 8));
-  MArgs a;
+  double* out = d_M;
+  if (ms.tiled) {
+    CSTF_TRY(w.partial.ensure((size_t)ms.Ivirt * R * 8));
+    out = w.partial.as<double>();
+  }
   a.rowptr = ms.rowptr.as<int64_t>();
   a.rec = ms.rec.as<char>();
   a.recb = ms.recb;
   a.nother = N - 1;
   for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
-  a.I = ms.I;
+  a.It = X->dims[ms.other[N - 2]];
+  a.I = ms.Ivirt;
   a.nnz = nnz;
   a.chunk = chunk;
   a.nchunks = nchunks;
   a.R = R;
   a.lb = w.lb.as<int64_t>();
   a.cont = w.cont.as<int32_t>();
-  a.M = d_M;
+  a.M = out;
   a.carry = w.carry.as<double>();
   if (ms.I == 0) return CSTF_OK;
+  int64_t nl = 0;
   {
     const int g = (int)std::min<int64_t>((nchunks + 1 + 255) / 256, (int64_t)di.sms * 8);
-    k_chunk_bounds<<<g, 256, 0, st>>>(a.rowptr, ms.I, nnz, chunk, nchunks, w.lb.as<int64_t>(),
+    k_chunk_bounds<<<g, 256, 0, st>>>(a.rowptr, ms.Ivirt, nnz, chunk, nchunks, a.wstart, w.lb.as<int64_t>(),
                                        w.cont.as<int32_t>());
     CSTF_LAUNCHED();
+    nl++;
   }
   const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
-  CSTF_TRY(launch_main(a, grid, st));
+  const int tgrid = (int)std::min<int64_t>(std::max<int64_t>(ms.nctachunks, 1), (int64_t)di.sms * 2);
+  CSTF_TRY(launch_main(a, grid, tgrid, st));
+  nl++;
   if (nchunks > 1) {
     const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);
-    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.carry, R, d_M);
+    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.carry, R, out);
     CSTF_LAUNCHED();
+    nl++;
   }
-  if (launches) *launches += (nchunks > 1) ? 3 : 2;
+  if (ms.tiled) {
+    const int64_t n = ms.I * R;
+    const int g = (int)std::min<int64_t>((n + 255) / 256, (int64_t)di.sms * 16);
+    k_reduce_blocks<<<g, 256, 0, st>>>(out, ms.I, ms.nblk, R, d_M);
+    CSTF_LAUNCHED();
+    nl++;
+  }
+  if (launches) *launches += nl;
   return CSTF_OK;
 }
 

@@ -10,6 +10,7 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "internal.h"
@@ -178,11 +179,12 @@ __global__ void k_histogram(const int32_t* __restrict__ key, int64_t n,
     atomicAdd(&cnt[key[p]], 1ull);
 }
 
-__global__ void k_expand_rows(const int64_t* __restrict__ rowptr, int64_t I,
+// out[p] = row of p (virtual row v -> v mod I)
+__global__ void k_expand_rows(const int64_t* __restrict__ rowptr, int64_t Iv, int64_t I,
                               int32_t* __restrict__ out) {
-  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < I;
-       i += (int64_t)gridDim.x * blockDim.x)
-    for (int64_t p = rowptr[i]; p < rowptr[i + 1]; p++) out[p] = (int32_t)i;
+  for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < Iv;
+       v += (int64_t)gridDim.x * blockDim.x)
+    for (int64_t p = rowptr[v]; p < rowptr[v + 1]; p++) out[p] = (int32_t)(v % I);
 }
 
 // Stable LSD radix sort of positions 0..n-1 by the key tuple keys[0..nk-1]
@@ -227,6 +229,16 @@ cstf_status lsd_sort(const int32_t* const* keys, const int64_t* dims, int nk, in
   }
   CSTF_CUDA(cudaStreamSynchronize(st));
   return CSTF_OK;
+}
+
+__global__ void k_block_keys(const int32_t* __restrict__ idx_t, const int32_t* __restrict__ idx_n, int64_t n,
+                             int64_t I, int32_t* __restrict__ kb, int32_t* __restrict__ vrow) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t b = idx_t[p] / kTileRows;
+    kb[p] = b;
+    vrow[p] = (int32_t)((int64_t)b * I + idx_n[p]);
+  }
 }
 
 struct RecArgs {
@@ -401,14 +413,32 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     for (int m = 0; m < N; m++)
       if (m != n_) ms.other[k++] = m;
     std::stable_sort(ms.other, ms.other + (N - 1), [&](int a, int b) { return X->dims[a] < X->dims[b]; });
-    const int32_t* keys[8];
-    int64_t kd[8];
-    keys[0] = c_idx[n_].as<int32_t>();
-    kd[0] = X->dims[n_];
-    for (int q = 0; q < N - 1; q++) { keys[q + 1] = c_idx[ms.other[q]].as<int32_t>(); kd[q + 1] = X->dims[ms.other[q]]; }
+    // k-blocking decision (host logic): short output mode, long other mode,
+    // enough nonzeros per partial row, bounded partial-row count
+    const int t = ms.other[N - 2];
+    const int64_t nblk = (X->dims[t] + kTileRows - 1) / kTileRows;
+    static const bool kblock_on = getenv("CSTF_KBLOCK") && atoi(getenv("CSTF_KBLOCK")) > 0;
+    ms.tiled = kblock_on && N >= 3 && nblk >= 2 && nblk * ms.I <= ((int64_t)4 << 20) && nout >= 8 * nblk * ms.I;
+    ms.nblk = ms.tiled ? nblk : 1;
+    ms.Ivirt = ms.nblk * ms.I;
+    const int32_t* keys[9];
+    int64_t kd[9];
+    int nk = 0;
+    DevBuf kbk, vrow;
+    if (ms.tiled) {
+      CSTF_TRY(kbk.alloc((size_t)nout * 4));
+      CSTF_TRY(vrow.alloc((size_t)nout * 4));
+      k_block_keys<<<grid_for(nout), kThreads, 0, st>>>(c_idx[t].as<int32_t>(), c_idx[n_].as<int32_t>(), nout,
+                                                        ms.I, kbk.as<int32_t>(), vrow.as<int32_t>());
+      CSTF_LAUNCHED();
+      keys[nk] = kbk.as<int32_t>(); kd[nk++] = nblk;
+    }
+    keys[nk] = c_idx[n_].as<int32_t>();
+    kd[nk++] = X->dims[n_];
+    for (int q = 0; q < N - 1; q++) { keys[nk] = c_idx[ms.other[q]].as<int32_t>(); kd[nk++] = X->dims[ms.other[q]]; }
     DevBuf pm;
-    CSTF_TRY(lsd_sort(keys, kd, N, nout, pm, tmp, st));
-    CSTF_TRY(build_rowptr(c_idx[n_].as<int32_t>(), nout, ms.I, ms.rowptr, tmp, st));
+    CSTF_TRY(lsd_sort(keys, kd, nk, nout, pm, tmp, st));
+    CSTF_TRY(build_rowptr(ms.tiled ? vrow.as<int32_t>() : c_idx[n_].as<int32_t>(), nout, ms.Ivirt, ms.rowptr, tmp, st));
     CSTF_TRY(ms.rec.alloc((size_t)nout * recb));
     RecArgs ra;
     ra.nslots = N - 1;
@@ -435,7 +465,8 @@ cstf_status export_store(const cstf_tensor* X, int32_t* const* host_idx, double*
   DevBuf soa[8], vals, tmp, perm, out;
   for (int m = 0; m < N; m++) CSTF_TRY(soa[m].alloc((size_t)n * 4));
   CSTF_TRY(vals.alloc((size_t)n * 8));
-  k_expand_rows<<<grid_for(ms.I), kThreads, 0, st>>>(ms.rowptr.as<int64_t>(), ms.I, soa[0].as<int32_t>());
+  k_expand_rows<<<grid_for(ms.Ivirt), kThreads, 0, st>>>(ms.rowptr.as<int64_t>(), ms.Ivirt, ms.I,
+                                                          soa[0].as<int32_t>());
   CSTF_LAUNCHED();
   OutArgs oa;
   oa.N = N - 1;

@@ -311,3 +311,31 @@ def test_factorize_host_matches_device(B):
     for a, b in zip(hf, F):
         assert np.array_equal(a, host(b))
     assert np.array_equal(hl, host(lam))
+
+
+@pytest.mark.parametrize("R", [8, 32, 5, 64])
+def test_mttkrp_kblocked_with_empty_blocks(B, R):
+    """k-blocked copies (short output mode, long other mode): blocks of the long
+    mode with no nonzeros still produce zero partial rows; rows absent from whole
+    blocks, heavy rows and empty output rows all match the oracle."""
+    rng = np.random.default_rng(R)
+    nnz = 60000
+    i = rng.integers(0, 40, nnz).astype(np.int32)
+    i[i == 13] = 14                                   # output row 13 empty
+    i[: nnz // 3] = 5                                 # a heavy output row
+    j = rng.integers(0, 30, nnz).astype(np.int32)
+    k = rng.integers(0, 2000, nnz).astype(np.int32)
+    k[(k >= 256) & (k < 1024)] += 1000               # blocks 1..3 of mode 2 empty
+    k = np.minimum(k, 1999).astype(np.int32)
+    dims = (40, 30, 2000)
+    vals = rng.random(nnz)
+    X = B.cstf_tensor_load_coo(dims, [i, j, k], vals)
+    ref = oracle.coalesce(dims, [i, j, k], vals)
+    gi, gv = X.export_coo()
+    assert np.array_equal(gv, ref.vals) and all(np.array_equal(a, b) for a, b in zip(gi, ref.idx))
+    F = [rng.random((I, R)) for I in dims]
+    Fd = [cu(f) for f in F]
+    for n in range(3):
+        M = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        assert normwise(host(M), oracle.mttkrp(ref, n, F)) <= TOL, n

@@ -7,25 +7,32 @@
 // B200 design:
 //  * Rows are independent; only the four sums couple them.  A warp owns 8 rows
 //    and keeps m, h, u in registers for ALL inner iterations of a launch
-//    (row-resident, "v2"): HBM traffic is 5 I R words per launch instead of
-//    per iteration.  One launch per iteration ("v1", streaming) uses the same
-//    code with kiters = 1.
+//    (row-resident): HBM traffic is 5 I R words per launch instead of per
+//    iteration.  One launch per iteration (streaming, the paper's shape) uses
+//    the same code with kiters = 1.
 //  * The R x R product runs on the FP64 tensor-core path: mma.sync m8n8k4 f64
 //    (SASS DMMA.8x8x4; tcgen05 has no f64 kind).  The accumulator (C) layout
 //    of the product is reused as the A operand of the next iteration by
 //    permuting the contraction index: thread (g = lane/4, q = lane%4) holds
 //    row g, columns {8t + 2q, 8t + 2q + 1}; A chunk c of that thread is column
-//    8(c/2) + 2q + (c%2), and the Inv fragment of chunk c is permuted the same
-//    way, so no shuffles are needed between iterations.
+//    8(c/2) + 2q + (c%2), and the Inv fragment of chunk c (in shared memory)
+//    is permuted the same way, so no shuffles are needed between iterations.
 //  * Per-iteration partial sums go to per-thread shared-memory slots and are
 //    reduced in fixed order per CTA, then over CTAs by a finalize kernel that
-//    also takes the stop decision on the device (deterministic).
+//    also takes the stop decision on the device (deterministic).  With
+//    tol = 0 the stop test is disabled by definition (exactly max_iter
+//    passes), so only the final pass's sums are formed (reported stats).
+//  * Optional epilogue: the Gram contribution H^T H of the final rows (still in
+//    registers) by 2 * NT(NT+1)/2 more DMMAs per 8 rows (Alg. 1 l.12 fused,
+//    R <= 32), and a per-column scale of M on load (lazy normalisation:
+//    M = M' diag(mscale)).
 #include "internal.h"
 
 namespace cstf {
 namespace {
 
 constexpr int kThreads = 128;   // 4 warps
+constexpr int kWarpsA = kThreads / 32;
 constexpr int kMaxK = 16;       // inner iterations per launch (chunk)
 
 struct KArgs {
@@ -35,6 +42,7 @@ struct KArgs {
   double* Hout;            // may alias H (in place) or be null (no write)
   double* Uout;
   const double* hscale;    // optional column scale of the incoming H
+  const double* mscale;    // optional column scale of M (lazy normalisation)
   int64_t I;
   int R;
   const double* inv;
@@ -42,7 +50,9 @@ struct KArgs {
   const int* flag;         // skip all work if a previous step failed
   int prox;
   int kiters;
+  int sums_from;           // first local pass whose residual sums are formed
   double* slots;           // [kiters][gridDim][4]
+  double* gpart;           // optional: per-CTA Gram partials [grid][NT(NT+1)/2][64]
 };
 
 __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b) {
@@ -51,46 +61,47 @@ __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b)
       : "d"(a), "d"(b));
 }
 
-// RP = padded rank (multiple of 8, <= 64).  INV_REGS: Inv fragments in registers (RP <= 32).
-template <int RP, bool INV_REGS>
+// RP = padded rank (multiple of 8, <= 64).  GRAM: fused Gram epilogue (RP <= 32).
+template <int RP, bool GRAM>
 __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
   constexpr int NT = RP / 8;       // n-tiles of 8 columns
   constexpr int NC = 2 * NT;       // k-chunks of 4
+  constexpr int NP = NT * (NT + 1) / 2;   // Gram tile pairs (a <= b)
   extern __shared__ double smem[];
-  double* sacc = smem;                                   // [kiters][4][kThreads]
-  double* sinv = smem + (size_t)kMaxK * 4 * kThreads;    // [NC][NT][32] fragments (if !INV_REGS)
+  const int nsl = a.kiters - a.sums_from;                // passes that form sums
+  double* sacc = smem;                                   // [nsl][4][kThreads]
+  double* sinv = smem + (size_t)nsl * 4 * kThreads;      // [NC][NT][32] Inv fragments
+  double* sg = sinv + (size_t)NC * NT * 32;              // [warp][NP][64] Gram tiles (GRAM)
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int g = lane >> 2, q = lane & 3;
   const int R = a.R;
   const bool skip = *a.flag != 0;   // an earlier step failed: write zero sums, touch nothing
   const double rho = a.scal[0];
   const int kiters = a.kiters;
-  for (int x = tid; x < kiters * 4 * kThreads; x += kThreads) sacc[x] = 0.0;
+  for (int x = tid; x < nsl * 4 * kThreads; x += kThreads) sacc[x] = 0.0;
+  if (GRAM)
+    for (int x = tid; x < kWarpsA * NP * 64; x += kThreads) sg[x] = 0.0;
   // B fragments: thread (g' = lane/4, q' = lane%4) holds Inv[kperm(c, q')][8t + g']
-  double binv[INV_REGS ? NC : 1][INV_REGS ? NT : 1];
-#pragma unroll
-  for (int c = 0; c < NC; c++)
-#pragma unroll
-    for (int t = 0; t < NT; t++) {
-      const int k = 8 * (c >> 1) + 2 * q + (c & 1);
-      const int n = 8 * t + g;
-      const double v = (k < R && n < R) ? a.inv[k * R + n] : 0.0;
-      if (INV_REGS) binv[INV_REGS ? c : 0][INV_REGS ? t : 0] = v;
-      else sinv[(c * NT + t) * 32 + lane] = v;
-    }
+  for (int x = tid; x < NC * NT * 32; x += kThreads) {
+    const int ln = x & 31, ct = x >> 5, c = ct / NT, t = ct % NT;
+    const int k = 8 * (c >> 1) + 2 * (ln & 3) + (c & 1);
+    const int n = 8 * t + (ln >> 2);
+    sinv[x] = (k < R && n < R) ? a.inv[k * R + n] : 0.0;
+  }
   __syncthreads();
-  double hs[NT][2];
+  double hs[NT][2], ms[NT][2];
 #pragma unroll
   for (int t = 0; t < NT; t++)
 #pragma unroll
     for (int i = 0; i < 2; i++) {
       const int col = 8 * t + 2 * q + i;
       hs[t][i] = (a.hscale && col < R) ? a.hscale[col] : 1.0;
+      ms[t][i] = (a.mscale && col < R) ? a.mscale[col] : 1.0;
     }
   const bool full = (R == RP);
   const int64_t ngroups = (a.I + 7) / 8;
-  const int64_t gw0 = (int64_t)blockIdx.x * (kThreads / 32) + warp;
-  const int64_t gws = (int64_t)gridDim.x * (kThreads / 32);
+  const int64_t gw0 = (int64_t)blockIdx.x * kWarpsA + warp;
+  const int64_t gws = (int64_t)gridDim.x * kWarpsA;
   for (int64_t grp = skip ? ngroups : gw0; grp < ngroups; grp += gws) {
     const int64_t row = grp * 8 + g;
     const bool rok = row < a.I;
@@ -117,7 +128,10 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
         }
       }
 #pragma unroll
-      for (int i = 0; i < 2; i++) h[t][i] = h[t][i] * hs[t][i];
+      for (int i = 0; i < 2; i++) {
+        h[t][i] = h[t][i] * hs[t][i];
+        m[t][i] = m[t][i] * ms[t][i];
+      }
     }
     for (int j = 0; j < kiters; j++) {
       double d[NT][2];
@@ -128,27 +142,63 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
         const int tt = c >> 1, ii = c & 1;
         const double av = fma(rho, h[tt][ii] + u[tt][ii], m[tt][ii]);   // M + rho (H + U)
 #pragma unroll
-        for (int t = 0; t < NT; t++) {
-          const double bv = INV_REGS ? binv[INV_REGS ? c : 0][INV_REGS ? t : 0] : sinv[(c * NT + t) * 32 + lane];
-          dmma(d[t][0], d[t][1], av, bv);
-        }
+        for (int t = 0; t < NT; t++) dmma(d[t][0], d[t][1], av, sinv[(c * NT + t) * 32 + lane]);
       }
-      double pr = 0.0, ps = 0.0, ph = 0.0, pu = 0.0;
+      if (j >= a.sums_from) {
+        double pr = 0.0, ps = 0.0, ph = 0.0, pu = 0.0;
 #pragma unroll
-      for (int t = 0; t < NT; t++)
+        for (int t = 0; t < NT; t++)
 #pragma unroll
-        for (int i = 0; i < 2; i++) {
-          const double ht = d[t][i];
-          const double x = ht - u[t][i];
-          const double hn = (a.prox == CSTF_PROX_IDENTITY) ? x : (x > 0.0 ? x : 0.0);
-          const double un = (u[t][i] + hn) - ht;
-          const double e1 = hn - ht, e2 = hn - h[t][i];
-          pr = fma(e1, e1, pr); ps = fma(e2, e2, ps); ph = fma(hn, hn, ph); pu = fma(un, un, pu);
-          h[t][i] = hn;
-          u[t][i] = un;
+          for (int i = 0; i < 2; i++) {
+            const double ht = d[t][i];
+            const double x = ht - u[t][i];
+            const double hn = (a.prox == CSTF_PROX_IDENTITY) ? x : (x > 0.0 ? x : 0.0);
+            const double un = (u[t][i] + hn) - ht;
+            const double e1 = hn - ht, e2 = hn - h[t][i];
+            pr = fma(e1, e1, pr); ps = fma(e2, e2, ps); ph = fma(hn, hn, ph); pu = fma(un, un, pu);
+            h[t][i] = hn;
+            u[t][i] = un;
+          }
+        double* sj = sacc + (size_t)(j - a.sums_from) * 4 * kThreads + tid;
+        sj[0] += pr; sj[kThreads] += ps; sj[2 * kThreads] += ph; sj[3 * kThreads] += pu;
+      } else {
+#pragma unroll
+        for (int t = 0; t < NT; t++)
+#pragma unroll
+          for (int i = 0; i < 2; i++) {
+            const double ht = d[t][i];
+            const double x = ht - u[t][i];
+            const double hn = (a.prox == CSTF_PROX_IDENTITY) ? x : (x > 0.0 ? x : 0.0);
+            u[t][i] = (u[t][i] + hn) - ht;
+            h[t][i] = hn;
+          }
+      }
+    }
+    if (GRAM) {
+      // fragment (x, kc) of both DMMA operands: H[row 4kc + q][col 8x + g], held by
+      // lane 4(4kc + q) + g/2 as element g%2 of its n-tile x
+      double fr[GRAM ? NT : 1][2];
+#pragma unroll
+      for (int x = 0; x < NT; x++)
+#pragma unroll
+        for (int kc = 0; kc < 2; kc++) {
+          const int src = 4 * (4 * kc + q) + (g >> 1);
+          const double v0 = __shfl_sync(0xffffffffu, h[x][0], src);
+          const double v1 = __shfl_sync(0xffffffffu, h[x][1], src);
+          fr[GRAM ? x : 0][kc] = (g & 1) ? v1 : v0;
         }
-      double* sj = sacc + (size_t)j * 4 * kThreads + tid;
-      sj[0] += pr; sj[kThreads] += ps; sj[2 * kThreads] += ph; sj[3 * kThreads] += pu;
+      int p = 0;
+      double* sgw = sg + (size_t)warp * NP * 64 + lane * 2;
+#pragma unroll
+      for (int xa = 0; xa < NT; xa++)
+#pragma unroll
+        for (int xb = xa; xb < NT; xb++, p++) {
+          double g0 = 0.0, g1 = 0.0;
+#pragma unroll
+          for (int kc = 0; kc < 2; kc++) dmma(g0, g1, fr[GRAM ? xa : 0][kc], fr[GRAM ? xb : 0][kc]);
+          sgw[p * 64] += g0;
+          sgw[p * 64 + 1] += g1;
+        }
     }
     if (a.Hout && rok) {
 #pragma unroll
@@ -167,17 +217,43 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
   }
   __syncthreads();
   // fixed-order CTA reduction of the per-thread slots
-  for (int x = tid; x < kiters * 4; x += kThreads) {
+  for (int x = tid; x < nsl * 4; x += kThreads) {
     const double* p = sacc + (size_t)x * kThreads;
     double s = 0.0;
     for (int k = 0; k < kThreads; k++) s += p[k];
-    const int j = x >> 2, w = x & 3;
+    const int j = a.sums_from + (x >> 2), w = x & 3;
     a.slots[((size_t)j * gridDim.x + blockIdx.x) * 4 + w] = s;
+  }
+  if (GRAM) {
+    for (int x = tid; x < NP * 64; x += kThreads) {
+      double s = 0.0;
+      for (int w = 0; w < kWarpsA; w++) s += sg[(size_t)w * NP * 64 + x];
+      a.gpart[(size_t)blockIdx.x * NP * 64 + x] = s;
+    }
   }
 }
 
-// Generic form for any R <= 128: one CTA row at a time, thread = column,
-// Inv column in registers-from-smem.  Same per-element arithmetic order.
+// G[a][b] (full R x R, raw) from the per-CTA tile partials of k_admm_dmma<RP, true>.
+// Element e = lane*2 + i of pair (xa, xb) is G[8 xa + lane/4][8 xb + 2 (lane%4) + i].
+__global__ void k_gram_from_parts(const double* __restrict__ gpart, int nblocks, int NT, int R,
+                                  double* __restrict__ G) {
+  const int NP = NT * (NT + 1) / 2;
+  for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < NP * 64; x += gridDim.x * blockDim.x) {
+    const int p = x / 64, e = x % 64, lane = e / 2, i = e % 2;
+    int xa = 0, rem = p;
+    while (rem >= NT - xa) { rem -= NT - xa; xa++; }
+    const int xb = xa + rem;
+    const int r = 8 * xa + lane / 4, c = 8 * xb + 2 * (lane % 4) + i;
+    if (r >= R || c >= R) continue;
+    if (xa == xb && r > c) continue;      // diagonal tile: upper triangle, mirrored
+    double s = 0.0;
+    for (int b = 0; b < nblocks; b++) s += gpart[(size_t)b * NP * 64 + x];
+    G[r * R + c] = s;
+    G[c * R + r] = s;
+  }
+}
+
+// Generic form for any R <= 128: one CTA row at a time, thread = column.
 __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
   extern __shared__ double smem[];
   double* sinv = smem;                       // [R][R]
@@ -193,9 +269,10 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
   __syncthreads();
   const bool cok = tid < R;
   const double hsc = (a.hscale && cok) ? a.hscale[tid] : 1.0;
+  const double msc = (a.mscale && cok) ? a.mscale[tid] : 1.0;
   for (int64_t row = skip ? a.I : blockIdx.x; row < a.I; row += gridDim.x) {
     const size_t base = (size_t)row * R;
-    double m = cok ? a.M[base + tid] : 0.0;
+    double m = cok ? a.M[base + tid] * msc : 0.0;
     double h = cok ? a.H[base + tid] * hsc : 0.0;
     double u = cok ? a.U[base + tid] : 0.0;
     for (int j = 0; j < kiters; j++) {
@@ -210,9 +287,11 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
       const double un = (u + hn) - ht;
       const double e1 = hn - ht, e2 = hn - h;
       if (cok) {
-        double* sj = sacc + (size_t)j * 4 * 128 + tid;
-        sj[0] = fma(e1, e1, sj[0]); sj[128] = fma(e2, e2, sj[128]);
-        sj[256] = fma(hn, hn, sj[256]); sj[384] = fma(un, un, sj[384]);
+        if (j >= a.sums_from) {
+          double* sj = sacc + (size_t)j * 4 * 128 + tid;
+          sj[0] = fma(e1, e1, sj[0]); sj[128] = fma(e2, e2, sj[128]);
+          sj[256] = fma(hn, hn, sj[256]); sj[384] = fma(un, un, sj[384]);
+        }
         h = hn;
         u = un;
       }
@@ -230,9 +309,9 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
 }
 
 // sums[j0 + j][w] = sum over CTAs (fixed order) of slots[j][cta][w]
-__global__ void k_admm_sum(const double* __restrict__ slots, int nblocks, int kiters, int j0,
+__global__ void k_admm_sum(const double* __restrict__ slots, int nblocks, int kiters, int from, int j0,
                            double* __restrict__ sums) {
-  for (int x = threadIdx.x; x < kiters * 4; x += blockDim.x) {
+  for (int x = threadIdx.x + from * 4; x < kiters * 4; x += blockDim.x) {
     const int j = x >> 2, w = x & 3;
     double s = 0.0;
     for (int b = 0; b < nblocks; b++) s += slots[((size_t)j * nblocks + b) * 4 + w];
@@ -241,8 +320,8 @@ __global__ void k_admm_sum(const double* __restrict__ slots, int nblocks, int ki
 }
 
 // Stop decision over iterations [j0, j0 + k): first j with r < tol nH and s < tol nU (D3),
-// or the last allowed iteration.  dec[0] = decided iteration count (0 = undecided),
-// dec[1] = flags (2 = non-finite).  stats out: iters, rho, r, s, nH, nU.
+// or the last allowed iteration.  out[0] = decided iteration count (0 = undecided),
+// out[1..5] = rho, r, s, nH, nU of that pass; flag |= 2 on non-finite sums.
 __global__ void k_admm_decide(const double* __restrict__ sums, int j0, int k, int max_iter, double tol,
                               const double* __restrict__ scal, int* __restrict__ flag,
                               double* __restrict__ out) {
@@ -269,7 +348,7 @@ __global__ void k_admm_decide(const double* __restrict__ sums, int j0, int k, in
 }
 
 struct Workspace {
-  DevBuf slots, sums, out, hs[2], us[2];
+  DevBuf slots, sums, out, hs[2], us[2], gpart;
   double* host_out = nullptr;
 };
 Workspace& ws() {
@@ -281,40 +360,54 @@ Workspace& ws() {
   return r;
 }
 
-template <int RP, bool REG>
-cstf_status launch_dmma_t(const KArgs& k, int grid, cudaStream_t st) {
-  const size_t smem = (size_t)kMaxK * 4 * kThreads * 8 + (REG ? 0 : (size_t)2 * (RP / 8) * (RP / 8) * 32 * 8);
+size_t dmma_smem(int RP, bool gram, int nsl) {
+  const int NT = RP / 8;
+  return (size_t)nsl * 4 * kThreads * 8 + (size_t)2 * NT * NT * 32 * 8 +
+         (gram ? (size_t)kWarpsA * NT * (NT + 1) / 2 * 64 * 8 : 0);
+}
+
+template <int RP, bool GRAM>
+cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
+  const int nsl = k.kiters - k.sums_from;
+  const size_t smem = dmma_smem(RP, GRAM, nsl);
+  static int per_sm[kMaxK + 1] = {0};
   static bool attr = false;
   if (!attr) {
-    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, REG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)dmma_smem(RP, GRAM, kMaxK)));
     attr = true;
   }
-  k_admm_dmma<RP, REG><<<grid, kThreads, smem, st>>>(k);
+  if (!per_sm[nsl]) {
+    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM>, kThreads, smem));
+    if (per_sm[nsl] < 1) per_sm[nsl] = 1;
+  }
+  const int64_t groups = (k.I + 7) / 8;
+  int64_t g = (groups + kWarpsA - 1) / kWarpsA;
+  const int64_t cap = (int64_t)device_info().sms * per_sm[nsl];
+  if (g > cap) g = cap;
+  grid = (int)(g < 1 ? 1 : g);
+  k_admm_dmma<RP, GRAM><<<grid, kThreads, smem, st>>>(k);
   CSTF_LAUNCHED();
   return CSTF_OK;
 }
 
-int grid_for_dmma(int RP, int64_t I) {
-  // persistent: up to (SMs x CTAs/SM); fewer when there are few row groups
-  const int sms = device_info().sms;
-  const int per_sm = RP <= 32 ? 3 : 2;
-  const int64_t groups = (I + 7) / 8;
-  int64_t g = (groups + 3) / 4;
-  int64_t cap = (int64_t)sms * per_sm;
-  if (g > cap) g = cap;
-  return (int)(g < 1 ? 1 : g);
-}
-
-cstf_status launch_kernel(const KArgs& k, int& grid, cudaStream_t st) {
+cstf_status launch_kernel(const KArgs& k, int& grid, bool gram, cudaStream_t st) {
   const int R = k.R;
   const int RP = (R + 7) & ~7;
   if (RP <= 64) {
-    grid = grid_for_dmma(RP, k.I);
+    if (gram) {
+      switch (RP) {
+        case 8: return launch_dmma_t<8, true>(k, grid, st);
+        case 16: return launch_dmma_t<16, true>(k, grid, st);
+        case 24: return launch_dmma_t<24, true>(k, grid, st);
+        case 32: return launch_dmma_t<32, true>(k, grid, st);
+      }
+    }
     switch (RP) {
-      case 8: return launch_dmma_t<8, true>(k, grid, st);
-      case 16: return launch_dmma_t<16, true>(k, grid, st);
-      case 24: return launch_dmma_t<24, true>(k, grid, st);
-      case 32: return launch_dmma_t<32, true>(k, grid, st);
+      case 8: return launch_dmma_t<8, false>(k, grid, st);
+      case 16: return launch_dmma_t<16, false>(k, grid, st);
+      case 24: return launch_dmma_t<24, false>(k, grid, st);
+      case 32: return launch_dmma_t<32, false>(k, grid, st);
       case 40: return launch_dmma_t<40, false>(k, grid, st);
       case 48: return launch_dmma_t<48, false>(k, grid, st);
       case 56: return launch_dmma_t<56, false>(k, grid, st);
@@ -336,10 +429,13 @@ cstf_status launch_kernel(const KArgs& k, int& grid, cudaStream_t st) {
 
 }  // namespace
 
+bool admm_can_fuse_gram(int R, double tol) { return tol == 0.0 && R <= 32; }
+
 // Runs one ADMM update.  tol == 0: chunks of up to kMaxK iterations in place,
-// no host round trip until the end.  tol > 0: each chunk runs speculatively
-// into scratch buffers, the device decides the stop iteration, and the chunk
-// is replayed exactly (same arithmetic) up to it when it ends early.
+// no host round trip until the end; the final chunk can also emit the Gram of
+// the result (A.G != null).  tol > 0: each chunk runs speculatively into
+// scratch buffers, the device decides the stop iteration, and the chunk is
+// replayed exactly (same arithmetic) up to it when it ends early.
 cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
                      cstf_admm_stats* stats, int* iters_out, int64_t* launches) {
   Workspace& w = ws();
@@ -347,12 +443,17 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
   const int64_t I = A.I;
   const int kchunk = (A.variant == CSTF_ADMM_STREAMING) ? 1 : kMaxK;
   const int maxgrid = device_info().sms * 8;
+  const bool spec = A.tol > 0.0;
+  const bool fuse_gram = A.G != nullptr && admm_can_fuse_gram(R, A.tol);
+  if (A.G && !fuse_gram) return fail(CSTF_ERR_INVALID_ARG, "fused Gram needs tol == 0 and R <= 32");
   CSTF_TRY(w.slots.ensure((size_t)kMaxK * maxgrid * 4 * 8));
   CSTF_TRY(w.sums.ensure((size_t)A.max_iter * 4 * 8));
   CSTF_TRY(w.out.ensure(16 * 8));
+  if (fuse_gram) CSTF_TRY(w.gpart.ensure((size_t)maxgrid * 10 * 64 * 8));
   int64_t nl = 0;
   KArgs k;
   k.M = A.M;
+  k.mscale = A.mscale;
   k.I = I;
   k.R = R;
   k.inv = A.inv;
@@ -360,7 +461,7 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
   k.flag = A.flag;
   k.prox = A.prox;
   k.slots = w.slots.as<double>();
-  const bool spec = A.tol > 0.0;
+  k.gpart = nullptr;
   if (spec) {
     for (int b = 0; b < 2; b++) {
       CSTF_TRY(w.hs[b].ensure((size_t)I * R * 8));
@@ -374,10 +475,14 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
   int decided = 0;
   for (int j0 = 0; j0 < A.max_iter;) {
     const int kk = std::min(kchunk, A.max_iter - j0);
+    const bool last = j0 + kk >= A.max_iter;
     k.H = curH;
     k.U = curU;
     k.hscale = cur_scale;
     k.kiters = kk;
+    k.sums_from = spec ? 0 : (last ? kk - 1 : kk);
+    const bool gram_now = fuse_gram && last;
+    k.gpart = gram_now ? w.gpart.as<double>() : nullptr;
     if (spec && kchunk > 1) {
       k.Hout = w.hs[pp].as<double>();
       k.Uout = w.us[pp].as<double>();
@@ -386,10 +491,16 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
       k.Uout = A.U;
     }
     int grid = 0;
-    CSTF_TRY(launch_kernel(k, grid, st));
-    k_admm_sum<<<1, 64, 0, st>>>(k.slots, grid, kk, j0, w.sums.as<double>());
+    CSTF_TRY(launch_kernel(k, grid, gram_now, st));
+    k_admm_sum<<<1, 64, 0, st>>>(k.slots, grid, kk, k.sums_from, j0, w.sums.as<double>());
     CSTF_LAUNCHED();
     nl += 2;
+    if (gram_now) {
+      const int NT = ((R + 7) & ~7) / 8;
+      k_gram_from_parts<<<(NT * (NT + 1) / 2 * 64 + 127) / 128, 128, 0, st>>>(w.gpart.as<double>(), grid, NT, R, A.G);
+      CSTF_LAUNCHED();
+      nl++;
+    }
     if (comm_nranks(comm) > 1) CSTF_TRY(comm_allreduce_f64(comm, w.sums.as<double>() + (size_t)j0 * 4, (size_t)kk * 4, st));
     if (!spec) {
       j0 += kk;
@@ -430,8 +541,10 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
       } else {                   // exact replay of the chunk up to the decided pass
         k.H = curH; k.U = curU; k.hscale = cur_scale;
         k.kiters = dj - j0;
+        k.sums_from = k.kiters;  // sums already known
+        k.gpart = nullptr;
         k.Hout = A.H; k.Uout = A.U;
-        CSTF_TRY(launch_kernel(k, grid, st));
+        CSTF_TRY(launch_kernel(k, grid, false, st));
         nl++;
       }
     }

@@ -91,7 +91,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
   CSTF_TRY(w.lam.ensure((size_t)N * R * 8));
   CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
-  CSTF_TRY(w.scal.ensure(64));
+  CSTF_TRY(w.scal.ensure((size_t)(8 + 2 * R) * 8));
   CSTF_TRY(w.flag.ensure(64));
   CSTF_TRY(w.fitbuf.ensure(300 * 8));
   CSTF_TRY(w.M.ensure((size_t)Imax * R * 8));
@@ -126,6 +126,14 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     if (rep->mode_launches) for (int p = 0; p < N * CSTF_NUM_PHASES; p++) rep->mode_launches[p] = 0;
     rep->outer_done = 0;
   }
+  // Lazy normalisation: d_factors hold the raw ADMM output
+  // H_raw = H^(n) diag(lambda^(n)); the normalised factor is never formed inside
+  // the loop.  MTTKRP of the raw factors is rescaled per column on the ADMM
+  // load (mscale = prod_{k != n} 1/lambda_k), the scaled warm start (D4) is
+  // H_raw itself, the Grams kept are those of the normalised factors, and the
+  // factors are normalised once at the end.
+  CSTF_TRY(w.scal.ensure((size_t)(8 + 2 * R) * 8));
+  double* colscale = w.scal.as<double>() + 8;           // [2R]: mscale, 1/lambda_n
   double fit_prev = 0.0;
   for (int t = 0; t < o->outer_iters; t++) {
     for (int n = 0; n < N; n++) {
@@ -133,35 +141,42 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       double* Gn = G + (size_t)n * R * R;
       // a1 + a3 + a4: S = *_{k!=n} G^(k), rho, Cholesky, Inv   (GRAM phase)
       tm.begin(n, CSTF_PHASE_GRAM);
-      CSTF_TRY(chol_inverse(nullptr, G, N, n, R, o->admm.rho, w.inv.as<double>(), w.scal.as<double>(), flag, st));
+      CSTF_TRY(chol_inverse(nullptr, G, N, n, R, o->admm.rho, w.inv.as<double>(), w.scal.as<double>(), flag, st,
+                            lam, colscale));
       tm.end(n, CSTF_PHASE_GRAM);
-      // a2: MTTKRP
+      // a2: MTTKRP of the raw factors
       tm.begin(n, CSTF_PHASE_MTTKRP);
       CSTF_TRY(mttkrp(X, n, R, d_factors, M, st, nullptr));
       tm.end(n, CSTF_PHASE_MTTKRP);
-      // a5: ADMM, warm start H^(n) diag(lambda^(n)) (D4) unless the literal reading
+      // a5: ADMM on M diag(mscale); warm start H_raw (D4) or the normalised H (literal)
       tm.begin(n, CSTF_PHASE_UPDATE);
       AdmmArgs a;
       a.M = M; a.H = d_factors[n]; a.U = U[n];
-      a.hscale = (o->warm == CSTF_WARM_SCALED) ? lam + n * R : nullptr;
+      a.mscale = colscale;
+      a.hscale = (o->warm == CSTF_WARM_SCALED) ? nullptr : colscale + R;
       a.I = I; a.R = R; a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
       a.tol = o->admm.tol; a.max_iter = o->admm.max_iter; a.prox = o->admm.prox; a.variant = o->admm.variant;
+      const bool fused = admm_can_fuse_gram(R, o->admm.tol);
+      a.G = fused ? Gn : nullptr;      // a7 fused into the ADMM epilogue
       int iters = 0;
       CSTF_TRY(admm_run(a, comm, st, nullptr, &iters, nullptr));
       if (rep && rep->admm_iters) rep->admm_iters[t * N + n] = iters;
       tm.end(n, CSTF_PHASE_UPDATE);
-      // a7: Gram of the update (raw), a6: lambda + normalisation (G scaled consistently)
-      tm.begin(n, CSTF_PHASE_GRAM);
-      CSTF_TRY(gram_raw(d_factors[n], I, R, Gn, st));
-      tm.end(n, CSTF_PHASE_GRAM);
+      // a7 (when not fused): raw Gram; a6: lambda and the normalised Gram
+      if (!fused) {
+        tm.begin(n, CSTF_PHASE_GRAM);
+        CSTF_TRY(gram_raw(d_factors[n], I, R, Gn, st));
+        tm.end(n, CSTF_PHASE_GRAM);
+      }
       tm.begin(n, CSTF_PHASE_NORMALIZE);
-      CSTF_TRY(normalize_from_gram(d_factors[n], I, R, Gn, lam + n * R, st));
+      CSTF_TRY(comm_allreduce_f64(comm, Gn, (size_t)R * R, st));
+      CSTF_TRY(gram_to_lambda(Gn, R, lam + n * R, st));
       tm.end(n, CSTF_PHASE_NORMALIZE);
     }
-    // a8: fit of [[lambda^(N); H]] with M of the last mode
+    // a8: fit of [[lambda^(N); H]]: inner product of M'(N) diag(mscale) with H_raw(N)
     tm.begin(N - 1, CSTF_PHASE_NORMALIZE);
     double* fb = w.fitbuf.as<double>();
-    CSTF_TRY(fit(X->normX2, X->dims[N - 1], R, M, d_factors[N - 1], lam + (N - 1) * R, G, N, fb + 4,
+    CSTF_TRY(fit(X->normX2, X->dims[N - 1], R, M, d_factors[N - 1], colscale, lam + (N - 1) * R, G, N, fb + 4,
                  fb, flag, comm, st));
     tm.end(N - 1, CSTF_PHASE_NORMALIZE);
     CSTF_CUDA(cudaMemcpyAsync(w.host_small, fb, 8, cudaMemcpyDeviceToHost, st));
@@ -175,6 +190,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     if (o->fit_tol > 0.0 && t > 0 && std::fabs(f - fit_prev) < o->fit_tol) break;
     fit_prev = f;
   }
+  // normalise the factors once (Alg. 1 l.11 applied to the final state)
+  for (int n = 0; n < N; n++) CSTF_TRY(scale_rows_by_cols(d_factors[n], X->dims[n], R, lam + n * R, 1, st));
   if (d_lambda)
     CSTF_CUDA(cudaMemcpyAsync(d_lambda, lam + (N - 1) * R, (size_t)R * 8, cudaMemcpyDeviceToDevice, st));
   CSTF_CUDA(cudaStreamSynchronize(st));

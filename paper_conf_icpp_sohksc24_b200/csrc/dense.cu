@@ -169,7 +169,21 @@ __global__ void k_fill(double* __restrict__ d, int64_t n, double v) {
 // L^-1 by column-parallel forward substitution, Inv = L^-T L^-1.
 __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __restrict__ grams,
                                int N, int skip, int R, double rho_in, double* __restrict__ Linv,
-                               double* __restrict__ Inv, double* __restrict__ scal, int* flag) {
+                               double* __restrict__ Inv, double* __restrict__ scal, int* flag,
+                               const double* __restrict__ lam, double* __restrict__ colscale) {
+  if (lam) {
+    for (int r = threadIdx.x; r < R; r += blockDim.x) {
+      double ms = 1.0;
+      for (int k = 0; k < N; k++) {
+        if (k == skip) continue;
+        const double l = lam[k * R + r];
+        ms = (l > 0.0) ? ms / l : 0.0;
+      }
+      colscale[r] = ms;
+      const double ls = lam[skip * R + r];
+      colscale[R + r] = (ls > 0.0) ? 1.0 / ls : 0.0;
+    }
+  }
   extern __shared__ double L[];  // [R][R]: A, then L in the lower triangle
   __shared__ double s_rho;
   __shared__ int s_bad;
@@ -247,14 +261,14 @@ __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __
 
 // fit: per block partial of sum_i sum_r M_ir H_ir lam_r
 __global__ void __launch_bounds__(256) k_fit_partial(const double* __restrict__ M, const double* __restrict__ H,
-                                                     const double* __restrict__ lam, int64_t I, int R,
+                                                     const double* __restrict__ colw, int64_t I, int R,
                                                      double* __restrict__ part) {
   __shared__ double sh[256];
   const int64_t n = I * R;
   double acc = 0.0;
   for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
        x += (int64_t)gridDim.x * blockDim.x)
-    acc = fma(M[x] * H[x], lam[x % R], acc);
+    acc = fma(M[x] * H[x], colw[x % R], acc);
   sh[threadIdx.x] = acc;
   __syncthreads();
   for (int s = 128; s > 0; s >>= 1) {
@@ -366,9 +380,15 @@ cstf_status gram_normalize(double* d_H, int64_t I, int R, double* d_G, double* d
   return CSTF_OK;
 }
 
+cstf_status gram_to_lambda(double* d_G, int R, double* d_lam, cudaStream_t st) {
+  k_gram_normalize<<<1, 1024, 0, st>>>(d_G, R, d_lam);
+  CSTF_LAUNCHED();
+  return CSTF_OK;
+}
+
 cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int skip, int R,
                          double rho_in, double* d_inv, double* d_scal, int* d_flag,
-                         cudaStream_t st) {
+                         cudaStream_t st, const double* d_lam, double* d_colscale) {
   Workspace& w = ws();
   CSTF_TRY(w.linv.ensure((size_t)R * R * 8));
   const size_t smem = (size_t)R * R * 8;
@@ -378,16 +398,16 @@ cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int sk
     attr_set = true;
   }
   k_chol_inverse<<<1, 256, smem, st>>>(d_S, d_grams, N, skip, R, rho_in, w.linv.as<double>(), d_inv,
-                                       d_scal, d_flag);
+                                       d_scal, d_flag, d_lam, d_colscale);
   CSTF_LAUNCHED();
   return CSTF_OK;
 }
 
 cstf_status fit(double normX2, int64_t I, int R, const double* d_M, const double* d_H,
-                const double* d_lam, const double* d_grams, int N, double* d_part, double* d_out,
-                int* d_flag, const cstf_comm* comm, cudaStream_t st) {
+                const double* d_colw, const double* d_lam, const double* d_grams, int N,
+                double* d_part, double* d_out, int* d_flag, const cstf_comm* comm, cudaStream_t st) {
   const int nb = 256;
-  k_fit_partial<<<nb, 256, 0, st>>>(d_M, d_H, d_lam, I, R, d_part);
+  k_fit_partial<<<nb, 256, 0, st>>>(d_M, d_H, d_colw, I, R, d_part);
   CSTF_LAUNCHED();
   k_fit_sum<<<1, 32, 0, st>>>(d_part, nb, d_out);
   CSTF_LAUNCHED();

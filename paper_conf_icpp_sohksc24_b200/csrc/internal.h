@@ -160,13 +160,19 @@ cstf_status fill(double* d, int64_t n, double v, cudaStream_t st);
 // One CTA: S = Hadamard of the Grams except `skip` (or copy of d_S when grams == nullptr),
 // rho, Cholesky of S + rho I, Inv = (S + rho I)^-1.  Writes d_inv (R x R), d_scal[0] = rho,
 // d_flag |= 1 on NOT_SPD.
+// With d_lam (N x R, lazy normalisation) also writes d_colscale[0..R) =
+// prod_{k != skip} 1/lambda_k (0 where lambda_k = 0) and d_colscale[R..2R) = 1/lambda_skip.
 cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int skip, int R,
                          double rho_in, double* d_inv, double* d_scal, int* d_flag,
-                         cudaStream_t st);
-// fit (D12): writes d_out[0] = fit; needs M of the last mode, its H, lam, all Grams.
+                         cudaStream_t st, const double* d_lam = nullptr, double* d_colscale = nullptr);
+// lambda_r = sqrt(G_rr); G <- D^-1 G D^-1 (H untouched)
+cstf_status gram_to_lambda(double* d_G, int R, double* d_lam, cudaStream_t st);
+// fit (D12): writes d_out[0] = fit.  inner = sum_i sum_r M_ir H_ir colw_r, xhat = lam^T (*G) lam.
+// (lazy normalisation: M = MTTKRP of the raw factors, H = raw last factor, colw = its mscale)
 cstf_status fit(double normX2, int64_t I, int R, const double* d_M, const double* d_H,
-                const double* d_lam, const double* d_grams, int N, double* d_part /* >= 256 */,
-                double* d_out /* [2] */, int* d_flag, const cstf_comm* comm, cudaStream_t st);
+                const double* d_colw, const double* d_lam, const double* d_grams, int N,
+                double* d_part /* >= 256 */, double* d_out /* [2] */, int* d_flag,
+                const cstf_comm* comm, cudaStream_t st);
 cstf_status scale_rows_by_cols(double* d_H, int64_t I, int R, const double* d_lam, int divide,
                                cudaStream_t st);
 
@@ -175,7 +181,9 @@ struct AdmmArgs {
   const double* M;
   double* H;
   double* U;
-  const double* hscale;  // optional per-column scale of the incoming H (warm start D4)
+  const double* hscale;  // optional per-column scale of the incoming H
+  const double* mscale = nullptr;  // optional per-column scale of M (lazy normalisation)
+  double* G = nullptr;   // optional: raw Gram H^T H of the result (fused epilogue)
   int64_t I;
   int R;
   const double* inv;     // device R x R
@@ -188,5 +196,6 @@ struct AdmmArgs {
 };
 cstf_status admm_run(const AdmmArgs& a, const cstf_comm* comm, cudaStream_t st,
                      cstf_admm_stats* stats, int* iters_out, int64_t* launches);
+bool admm_can_fuse_gram(int R, double tol);
 
 }  // namespace cstf

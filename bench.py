@@ -159,15 +159,17 @@ def main():
     rank, world, local = env_rank()
     torch.cuda.set_device(local)
     dist = None
+    comm = None
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        comm = B.cstf_comm_create_nccl()     # rows of every mode partitioned over the ranks
     R = cfg.R
     t0 = time.time()
     idx, vals = cfg.generate()
     t_gen = time.time() - t0
     t0 = time.time()
-    X = B.cstf_tensor_load_coo(cfg.dims, idx, vals)
+    X = B.cstf_tensor_load_coo(cfg.dims, idx, vals, comm=comm)
     torch.cuda.synchronize()
     t_load = time.time() - t0
     info = X.info()
@@ -180,7 +182,7 @@ def main():
         return B.make_opts(R, outer_iters=n, tol=0.0, max_iter=10, timing=timing)
 
     # warm-up: W outer iterations
-    B.cstf_factorize(X, F, lam, opts(max(args.warmup, 3)))
+    B.cstf_factorize(X, F, lam, opts(max(args.warmup, 3)), comm=comm)
     torch.cuda.synchronize()
     # timed: K outer iterations in one call (each call starts with the init pass: included)
     clocks = ClockSampler(local)
@@ -191,7 +193,7 @@ def main():
     l0 = B.cstf_kernel_launch_count()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
-    rep = B.cstf_factorize(X, F, lam, opts(args.steps, timing=True))
+    rep = B.cstf_factorize(X, F, lam, opts(args.steps, timing=True), comm=comm)
     e1.record(stream)
     torch.cuda.synchronize()
     launches = B.cstf_kernel_launch_count() - l0
@@ -246,7 +248,7 @@ def main():
     if not args.no_e2e:
         hf = [torch.from_numpy(f.copy()).pin_memory() for f in F0]
         hl = torch.zeros(R, dtype=torch.float64).pin_memory()
-        B.cstf_factorize_host(X, hf, hl, opts(1))
+        B.cstf_factorize_host(X, hf, hl, opts(1), comm=comm)
         ts = []
         for _ in range(K):
             for h, f in zip(hf, F0):
@@ -254,7 +256,7 @@ def main():
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             torch.cuda.synchronize()
             a.record(stream)
-            B.cstf_factorize_host(X, hf, hl, opts(1))
+            B.cstf_factorize_host(X, hf, hl, opts(1), comm=comm)
             b.record(stream)
             torch.cuda.synchronize()
             ts.append(a.elapsed_time(b))

@@ -77,6 +77,9 @@ _decl("cstf_kernel_launch_count", c_int64, [])
 _decl("cstf_get_unique_id", c_int, [c_void_p])
 _decl("cstf_comm_create", c_int, [c_int, c_int, c_void_p, ctypes.POINTER(c_void_p)])
 _decl("cstf_comm_info", c_int, [c_void_p, ctypes.POINTER(c_int), ctypes.POINTER(c_int)])
+_ALLREDUCE_FN = ctypes.CFUNCTYPE(c_int, ctypes.POINTER(c_double), c_int64, c_void_p)
+_ALLGATHER_FN = ctypes.CFUNCTYPE(c_int, ctypes.POINTER(c_double), ctypes.POINTER(c_double), c_int64, c_void_p)
+_decl("cstf_comm_create_host", c_int, [c_int, c_int, _ALLREDUCE_FN, _ALLGATHER_FN, c_void_p, ctypes.POINTER(c_void_p)])
 _decl("cstf_comm_destroy", None, [c_void_p])
 _decl("cstf_partition_rows", c_int, [c_int64, c_void_p, c_int, c_void_p, c_void_p])
 _decl("cstf_tensor_load_coo", c_int, [c_int, c_void_p, c_int64, c_void_p, c_void_p, c_void_p, c_void_p,
@@ -96,7 +99,8 @@ _decl("cstf_factorize_host", c_int, [c_void_p, ctypes.POINTER(Opts), c_void_p, c
                                      ctypes.POINTER(Report), c_void_p])
 
 EXPORTED = ["cstf_status_string", "cstf_last_error_message", "cstf_version", "cstf_get_unique_id",
-            "cstf_comm_create", "cstf_comm_info", "cstf_comm_destroy", "cstf_partition_rows",
+            "cstf_comm_create", "cstf_comm_create_host", "cstf_comm_info", "cstf_comm_destroy",
+            "cstf_partition_rows",
             "cstf_tensor_load_coo", "cstf_tensor_info", "cstf_tensor_export_coo", "cstf_tensor_free",
             "cstf_mttkrp", "cstf_gram", "cstf_normalize", "cstf_admm_update", "cstf_factorize",
             "cstf_factorize_host", "cstf_kernel_launch_count"]
@@ -164,6 +168,53 @@ class Comm:
         if getattr(self, "handle", None):
             _lib.cstf_comm_destroy(self.handle)
             self.handle = None
+
+
+def cstf_comm_create_host(group=None) -> Comm:
+    """Host-callback communicator over a torch.distributed process group (e.g.
+    gloo): lets several processes share one GPU (NCCL needs one GPU per rank).
+    The library stages device buffers through host memory; the callbacks only
+    move bytes (sum / concatenate) through the process group."""
+    import torch
+    import torch.distributed as dist
+    P = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+
+    def allreduce(buf, n, user):
+        try:
+            t = torch.from_numpy(np.ctypeslib.as_array(buf, shape=(n,)))
+            dist.all_reduce(t, group=group)
+            return 0
+        except Exception:
+            return 1
+
+    def allgather(send, recv, n, user):
+        try:
+            s = torch.from_numpy(np.ctypeslib.as_array(send, shape=(n,)).copy())
+            r = torch.from_numpy(np.ctypeslib.as_array(recv, shape=(n * P,)))
+            dist.all_gather(list(r.chunk(P)), s, group=group)
+            return 0
+        except Exception:
+            return 1
+
+    cb = (_ALLREDUCE_FN(allreduce), _ALLGATHER_FN(allgather))
+    h = c_void_p()
+    _check(_lib.cstf_comm_create_host(P, rank, cb[0], cb[1], None, ctypes.byref(h)), "cstf_comm_create_host")
+    c = Comm(h.value)
+    c._callbacks = cb          # keep the trampolines alive
+    return c
+
+
+def cstf_comm_create_nccl(group=None) -> Comm:
+    """NCCL communicator (one process per GPU); the unique id travels through the
+    torch.distributed process group."""
+    import torch
+    import torch.distributed as dist
+    P = dist.get_world_size(group)
+    rank = dist.get_rank(group)
+    uid = [cstf_get_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(uid, src=0, group=group)
+    return cstf_comm_create(P, rank, uid[0])
 
 
 def cstf_get_unique_id() -> bytes:

@@ -501,7 +501,9 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
       CSTF_LAUNCHED();
       nl++;
     }
-    if (comm_nranks(comm) > 1) CSTF_TRY(comm_allreduce_f64(comm, w.sums.as<double>() + (size_t)j0 * 4, (size_t)kk * 4, st));
+    if (comm_nranks(comm) > 1 && kk > k.sums_from)   // every rank then takes the same stop decision
+      CSTF_TRY(comm_allreduce_f64(comm, w.sums.as<double>() + (size_t)(j0 + k.sums_from) * 4,
+                                  (size_t)(kk - k.sums_from) * 4, st));
     if (!spec) {
       j0 += kk;
       curH = A.H; curU = A.U; cur_scale = nullptr;

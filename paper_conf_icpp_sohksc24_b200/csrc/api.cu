@@ -10,11 +10,32 @@ namespace {
 
 cudaStream_t S(void* s) { return static_cast<cudaStream_t>(s); }
 
+// dst[lab[i]] = src[i] (to_internal) or dst[i] = src[lab[i]] (from internal), rows of R doubles
+__global__ void k_relabel_rows(const double* __restrict__ src, const int32_t* __restrict__ lab, int64_t I, int R,
+                               double* __restrict__ dst, int to_internal) {
+  const int64_t n = I * R;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = x / R, c = x % R;
+    const int64_t l = lab[i];
+    if (to_internal) dst[l * R + c] = src[x];
+    else dst[x] = src[l * R + c];
+  }
+}
+
+cstf_status relabel_rows(const double* src, const int32_t* lab, int64_t I, int R, double* dst, int to_internal,
+                         cudaStream_t st) {
+  if (I * R == 0) return CSTF_OK;
+  const int g = (int)std::min<int64_t>((I * R + 255) / 256, (int64_t)device_info().sms * 16);
+  k_relabel_rows<<<g, 256, 0, st>>>(src, lab, I, R, dst, to_internal);
+  CSTF_LAUNCHED();
+  return CSTF_OK;
+}
+
 bool rank_ok(int R) { return R >= 1 && R <= 128; }
 
 // Device-side scratch of one factorize / admm_update call, cached per device.
 struct DriverWs {
-  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac;
+  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8];
   double* host_small = nullptr;  // pinned: fit, flags
 };
 DriverWs& dws() {
@@ -82,12 +103,35 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   const int R = o->R;
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
   if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
-  if (comm_nranks(comm) > 1) return fail(CSTF_ERR_UNSUPPORTED, "distributed factorize: use a partitioned tensor");
+  const bool dist = X->nranks > 1;
+  if (comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
+    return fail(CSTF_ERR_INVALID_ARG, "comm does not match the tensor's partition");
   for (int n = 0; n < N; n++)
     if (!d_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");
   DriverWs& w = dws();
+  // Distributed: every rank keeps full factors in the
+  // internal (relabelled, zero-padded) row order; its own rows are the slice
+  // [rank*B_n, (rank+1)*B_n).  Single GPU: the caller's buffers, all rows local.
+  std::vector<double*> fac(N);
+  std::vector<int64_t> Ifull(N), Iloc(N), off(N);
+  for (int n = 0; n < N; n++) {
+    if (dist) {
+      const int64_t B = X->rows_per_rank[n];
+      Ifull[n] = (int64_t)X->nranks * B;
+      Iloc[n] = B;
+      off[n] = (int64_t)X->rank * B * R;
+      CSTF_TRY(w.Fi[n].ensure((size_t)Ifull[n] * R * 8));
+      fac[n] = w.Fi[n].as<double>();
+      CSTF_CUDA(cudaMemsetAsync(fac[n], 0, (size_t)Ifull[n] * R * 8, st));
+      CSTF_TRY(relabel_rows(d_factors[n], X->relabel[n].as<int32_t>(), X->dims[n], R, fac[n], 1, st));
+    } else {
+      Ifull[n] = Iloc[n] = X->dims[n];
+      off[n] = 0;
+      fac[n] = d_factors[n];
+    }
+  }
   int64_t Imax = 0, Usum = 0;
-  for (int n = 0; n < N; n++) { Imax = std::max(Imax, X->dims[n]); Usum += X->dims[n] * R; }
+  for (int n = 0; n < N; n++) { Imax = std::max(Imax, Iloc[n]); Usum += Iloc[n] * R; }
   CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
   CSTF_TRY(w.lam.ensure((size_t)N * R * 8));
   CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
@@ -103,15 +147,15 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   std::vector<double*> U(N);
   {
     int64_t off = 0;
-    for (int n = 0; n < N; n++) { U[n] = w.U.as<double>() + off; off += X->dims[n] * R; }
+    for (int n = 0; n < N; n++) { U[n] = w.U.as<double>() + off; off += Iloc[n] * R; }
   }
   CSTF_CUDA(cudaMemsetAsync(flag, 0, 4, st));
   CSTF_CUDA(cudaMemsetAsync(w.U.p, 0, (size_t)Usum * 8, st));
   // init (Alg. 1 l.1-5; readings D6): normalise, lambda = 1, G = H^T H
-  for (int n = 0; n < N; n++) {
+  for (int n = 0; n < N; n++) {      // factors are replicated: redundant, no communication
     double* Gn = G + (size_t)n * R * R;
-    CSTF_TRY(gram_raw(d_factors[n], X->dims[n], R, Gn, st));
-    if (o->normalize_init) CSTF_TRY(normalize_from_gram(d_factors[n], X->dims[n], R, Gn, lam + n * R, st));
+    CSTF_TRY(gram_raw(fac[n], Ifull[n], R, Gn, st));
+    if (o->normalize_init) CSTF_TRY(normalize_from_gram(fac[n], Ifull[n], R, Gn, lam + n * R, st));
     CSTF_TRY(fill(lam + n * R, R, 1.0, st));
   }
   PhaseTimer tm;
@@ -137,7 +181,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   double fit_prev = 0.0;
   for (int t = 0; t < o->outer_iters; t++) {
     for (int n = 0; n < N; n++) {
-      const int64_t I = X->dims[n];
+      const int64_t I = Iloc[n];
+      double* Hn = fac[n] + off[n];     // this rank's rows of the raw factor
       double* Gn = G + (size_t)n * R * R;
       // a1 + a3 + a4: S = *_{k!=n} G^(k), rho, Cholesky, Inv   (GRAM phase)
       tm.begin(n, CSTF_PHASE_GRAM);
@@ -146,12 +191,12 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       tm.end(n, CSTF_PHASE_GRAM);
       // a2: MTTKRP of the raw factors
       tm.begin(n, CSTF_PHASE_MTTKRP);
-      CSTF_TRY(mttkrp(X, n, R, d_factors, M, st, nullptr));
+      CSTF_TRY(mttkrp(X, n, R, fac.data(), M, st, nullptr));
       tm.end(n, CSTF_PHASE_MTTKRP);
       // a5: ADMM on M diag(mscale); warm start H_raw (D4) or the normalised H (literal)
       tm.begin(n, CSTF_PHASE_UPDATE);
       AdmmArgs a;
-      a.M = M; a.H = d_factors[n]; a.U = U[n];
+      a.M = M; a.H = Hn; a.U = U[n];
       a.mscale = colscale;
       a.hscale = (o->warm == CSTF_WARM_SCALED) ? nullptr : colscale + R;
       a.I = I; a.R = R; a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
@@ -165,8 +210,13 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       // a7 (when not fused): raw Gram; a6: lambda and the normalised Gram
       if (!fused) {
         tm.begin(n, CSTF_PHASE_GRAM);
-        CSTF_TRY(gram_raw(d_factors[n], I, R, Gn, st));
+        CSTF_TRY(gram_raw(Hn, I, R, Gn, st));
         tm.end(n, CSTF_PHASE_GRAM);
+      }
+      if (dist) {                        // every rank needs the updated factor for the next MTTKRPs
+        tm.begin(n, CSTF_PHASE_COMM);
+        CSTF_TRY(comm_allgather_f64(comm, Hn, fac[n], (size_t)I * R, st));
+        tm.end(n, CSTF_PHASE_COMM);
       }
       tm.begin(n, CSTF_PHASE_NORMALIZE);
       CSTF_TRY(comm_allreduce_f64(comm, Gn, (size_t)R * R, st));
@@ -176,7 +226,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     // a8: fit of [[lambda^(N); H]]: inner product of M'(N) diag(mscale) with H_raw(N)
     tm.begin(N - 1, CSTF_PHASE_NORMALIZE);
     double* fb = w.fitbuf.as<double>();
-    CSTF_TRY(fit(X->normX2, X->dims[N - 1], R, M, d_factors[N - 1], colscale, lam + (N - 1) * R, G, N, fb + 4,
+    CSTF_TRY(fit(X->normX2, Iloc[N - 1], R, M, fac[N - 1] + off[N - 1], colscale, lam + (N - 1) * R, G, N, fb + 4,
                  fb, flag, comm, st));
     tm.end(N - 1, CSTF_PHASE_NORMALIZE);
     CSTF_CUDA(cudaMemcpyAsync(w.host_small, fb, 8, cudaMemcpyDeviceToHost, st));
@@ -191,7 +241,10 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     fit_prev = f;
   }
   // normalise the factors once (Alg. 1 l.11 applied to the final state)
-  for (int n = 0; n < N; n++) CSTF_TRY(scale_rows_by_cols(d_factors[n], X->dims[n], R, lam + n * R, 1, st));
+  for (int n = 0; n < N; n++) {
+    CSTF_TRY(scale_rows_by_cols(fac[n], Ifull[n], R, lam + n * R, 1, st));
+    if (dist) CSTF_TRY(relabel_rows(fac[n], X->relabel[n].as<int32_t>(), X->dims[n], R, d_factors[n], 0, st));
+  }
   if (d_lambda)
     CSTF_CUDA(cudaMemcpyAsync(d_lambda, lam + (N - 1) * R, (size_t)R * 8, cudaMemcpyDeviceToDevice, st));
   CSTF_CUDA(cudaStreamSynchronize(st));
@@ -215,9 +268,10 @@ cstf_status cstf_tensor_load_coo(int nmodes, const int64_t* dims, int64_t nnz,
     if (dims[n] < 1 || dims[n] > 2147483647LL) return fail(CSTF_ERR_INVALID_ARG, "dims[n] must be in [1, 2^31-1]");
     if (nnz > 0 && !host_idx[n]) return fail(CSTF_ERR_INVALID_ARG, "host_idx[n] is NULL");
   }
-  if (comm_nranks(comm) > 1) return fail(CSTF_ERR_UNSUPPORTED, "partitioned load not built yet");
   cstf_tensor* X = new cstf_tensor();
   X->N = nmodes;
+  X->nranks = comm_nranks(comm);
+  X->rank = comm_rank(comm);
   for (int n = 0; n < nmodes; n++) X->dims[n] = dims[n];
   cudaGetDevice(&X->device);
   cstf_status s = build_store(X, host_idx, host_vals, nnz, S(stream));
@@ -249,6 +303,7 @@ cstf_status cstf_mttkrp(const cstf_tensor* X, int mode, int R, const double* con
                         void* stream) {
   if (!X || !d_factors || !d_M) return fail(CSTF_ERR_INVALID_ARG, "NULL argument");
   if (mode < 0 || mode >= X->N) return fail(CSTF_ERR_INVALID_ARG, "mode out of range");
+  if (X->nranks > 1) return fail(CSTF_ERR_UNSUPPORTED, "cstf_mttkrp on a partitioned tensor (use cstf_factorize)");
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
   for (int k = 0; k < X->N; k++)
     if (k != mode && !d_factors[k]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");

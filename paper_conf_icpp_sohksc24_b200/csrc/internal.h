@@ -76,6 +76,9 @@ struct Comm {
   int nranks = 1;
   int rank = 0;
   void* nccl = nullptr;  // ncclComm_t
+  cstf_host_allreduce_fn host_allreduce = nullptr;   // host-callback transport
+  cstf_host_allgather_fn host_allgather = nullptr;
+  void* user = nullptr;
 };
 cstf_status comm_allreduce_f64(const cstf_comm* c, double* d_buf, size_t count, cudaStream_t st);
 cstf_status comm_allgather_f64(const cstf_comm* c, const double* d_send, double* d_recv,
@@ -128,11 +131,13 @@ struct cstf_tensor {
   uint64_t hash = 0;
   int device = -1;
   cstf::ModeStore mode[8];
-  // distributed layout (nranks > 1): relabel maps original -> internal label
+  // distributed layout (nranks > 1): rows of mode n are dealt to ranks
+  // (cstf_partition_rows); internal label of row i = owner(i) * B_n + local(i),
+  // so every rank's rows are one contiguous slice [rank*B_n, (rank+1)*B_n) of the
+  // internal (relabelled, zero-padded) factor of P*B_n rows.
   int nranks = 1, rank = 0;
-  int64_t rows_per_rank[8] = {0};     // block size per rank (padded), per mode
+  int64_t rows_per_rank[8] = {0};     // B_n
   cstf::DevBuf relabel[8];            // int32[dims[n]]: internal label of original row
-  cstf::DevBuf unlabel[8];            // int32[nranks*rows_per_rank]: original row (or -1 pad)
 };
 
 namespace cstf {

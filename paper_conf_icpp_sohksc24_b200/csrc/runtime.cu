@@ -116,6 +116,16 @@ int comm_rank(const cstf_comm* c) { return c ? c->c.rank : 0; }
 
 cstf_status comm_allreduce_f64(const cstf_comm* c, double* d_buf, size_t count, cudaStream_t st) {
   if (!c || c->c.nranks <= 1 || count == 0) return CSTF_OK;
+  if (c->c.host_allreduce) {
+    std::vector<double> h(count);
+    CSTF_CUDA(cudaMemcpyAsync(h.data(), d_buf, count * 8, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    if (c->c.host_allreduce(h.data(), (int64_t)count, c->c.user) != 0)
+      return fail(CSTF_ERR_NCCL, "host all-reduce callback failed");
+    CSTF_CUDA(cudaMemcpyAsync(d_buf, h.data(), count * 8, cudaMemcpyHostToDevice, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    return CSTF_OK;
+  }
   return nccl_check(g_nccl.AllReduce(d_buf, d_buf, count, ncclFloat64, ncclSum,
                                      (ncclComm_t)c->c.nccl, st), "ncclAllReduce");
 }
@@ -124,6 +134,17 @@ cstf_status comm_allgather_f64(const cstf_comm* c, const double* d_send, double*
   if (!c || c->c.nranks <= 1) {
     if (d_send != d_recv && count_per_rank)
       CSTF_CUDA(cudaMemcpyAsync(d_recv, d_send, count_per_rank * 8, cudaMemcpyDeviceToDevice, st));
+    return CSTF_OK;
+  }
+  if (c->c.host_allgather) {
+    const size_t P = (size_t)c->c.nranks;
+    std::vector<double> hs(count_per_rank), hr(count_per_rank * P);
+    CSTF_CUDA(cudaMemcpyAsync(hs.data(), d_send, count_per_rank * 8, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    if (c->c.host_allgather(hs.data(), hr.data(), (int64_t)count_per_rank, c->c.user) != 0)
+      return fail(CSTF_ERR_NCCL, "host all-gather callback failed");
+    CSTF_CUDA(cudaMemcpyAsync(d_recv, hr.data(), hr.size() * 8, cudaMemcpyHostToDevice, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
     return CSTF_OK;
   }
   return nccl_check(g_nccl.AllGather(d_send, d_recv, count_per_rank, ncclFloat64,
@@ -181,6 +202,20 @@ cstf_status cstf_comm_create(int nranks, int rank, const unsigned char id[128], 
     if (s != CSTF_OK) { delete c; return s; }
     c->c.nccl = nc;
   }
+  *out = c;
+  return CSTF_OK;
+}
+
+cstf_status cstf_comm_create_host(int nranks, int rank, cstf_host_allreduce_fn allreduce,
+                                  cstf_host_allgather_fn allgather, void* user, cstf_comm** out) {
+  if (!out || nranks < 1 || rank < 0 || rank >= nranks || !allreduce || !allgather)
+    return fail(CSTF_ERR_INVALID_ARG, "cstf_comm_create_host arguments");
+  cstf_comm* c = new cstf_comm();
+  c->c.nranks = nranks;
+  c->c.rank = rank;
+  c->c.host_allreduce = allreduce;
+  c->c.host_allgather = allgather;
+  c->c.user = user;
   *out = c;
   return CSTF_OK;
 }

@@ -12,6 +12,7 @@
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
+#include <vector>
 
 #include "internal.h"
 
@@ -241,6 +242,35 @@ __global__ void k_block_keys(const int32_t* __restrict__ idx_t, const int32_t* _
   }
 }
 
+// out[p] = lab[in[p]]
+__global__ void k_map(const int32_t* __restrict__ in, const int32_t* __restrict__ lab, int64_t n,
+                      int32_t* __restrict__ out) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    out[p] = lab[in[p]];
+}
+
+// positions p whose internal row label falls in [lo, hi) (stable compaction: count + scan + scatter)
+__global__ void k_flag_range(const int32_t* __restrict__ lab, int64_t n, int32_t lo, int32_t hi,
+                             uint32_t* __restrict__ flag) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    flag[p] = (lab[p] >= lo && lab[p] < hi) ? 1u : 0u;
+}
+__global__ void k_scatter_sel(const uint32_t* __restrict__ flag, const uint32_t* __restrict__ incl, int64_t n,
+                              uint32_t* __restrict__ sel) {
+  for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
+       p += (int64_t)gridDim.x * blockDim.x)
+    if (flag[p]) sel[incl[p] - 1] = (uint32_t)p;
+}
+// out[s] = in[sel[s]] - shift
+__global__ void k_gather_shift(const int32_t* __restrict__ in, const uint32_t* __restrict__ sel, int64_t n,
+                               int32_t shift, int32_t* __restrict__ out) {
+  for (int64_t s = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; s < n;
+       s += (int64_t)gridDim.x * blockDim.x)
+    out[s] = in[sel[s]] - shift;
+}
+
 struct RecArgs {
   const int32_t* idx[7];   // slot q source index array (canonical order)
   int nslots;
@@ -296,6 +326,123 @@ cstf_status build_rowptr(const int32_t* d_key, int64_t n, int64_t I, DevBuf& row
 }
 
 }  // namespace
+
+// Partitioned copies: rows of every mode are dealt to
+// ranks (cstf_partition_rows); all indices are relabelled to
+// owner * B_n + local, and this rank keeps, for every mode n, the nonzeros whose
+// mode-n row it owns, with the row index local to its block.
+cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int64_t nout, DevBuf& tmp,
+                              cudaStream_t st) {
+  const int N = X->N, P = X->nranks, rk = X->rank;
+  DevBuf lab_idx[8];
+  for (int n = 0; n < N; n++) {
+    const int64_t I = X->dims[n];
+    DevBuf cnt;
+    CSTF_TRY(cnt.alloc((size_t)I * 8));
+    CSTF_CUDA(cudaMemsetAsync(cnt.p, 0, (size_t)I * 8, st));
+    if (nout) {
+      k_histogram<<<grid_for(nout), kThreads, 0, st>>>(c_idx[n].as<int32_t>(), nout, cnt.as<unsigned long long>());
+      CSTF_LAUNCHED();
+    }
+    std::vector<int64_t> counts((size_t)I), local((size_t)I);
+    std::vector<int32_t> owner((size_t)I), lab((size_t)I);
+    CSTF_CUDA(cudaMemcpyAsync(counts.data(), cnt.p, (size_t)I * 8, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    CSTF_TRY(cstf_partition_rows(I, counts.data(), P, owner.data(), local.data()));
+    const int64_t B = (I + P - 1) / P;
+    if ((int64_t)P * B >= ((int64_t)1 << 31)) return fail(CSTF_ERR_UNSUPPORTED, "padded mode length >= 2^31");
+    X->rows_per_rank[n] = B;
+    for (int64_t i = 0; i < I; i++) lab[(size_t)i] = (int32_t)(owner[(size_t)i] * B + local[(size_t)i]);
+    CSTF_TRY(X->relabel[n].alloc((size_t)I * 4));
+    CSTF_CUDA(cudaMemcpyAsync(X->relabel[n].p, lab.data(), (size_t)I * 4, cudaMemcpyHostToDevice, st));
+    CSTF_TRY(lab_idx[n].alloc((size_t)nout * 4));
+    if (nout) {
+      k_map<<<grid_for(nout), kThreads, 0, st>>>(c_idx[n].as<int32_t>(), X->relabel[n].as<int32_t>(), nout,
+                                                lab_idx[n].as<int32_t>());
+      CSTF_LAUNCHED();
+    }
+    CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  const int recb = record_bytes(N);
+  for (int n = 0; n < N; n++) {
+    ModeStore& ms = X->mode[n];
+    const int64_t B = X->rows_per_rank[n];
+    ms.I = B;
+    ms.Ivirt = B;
+    ms.tiled = false;
+    ms.nblk = 1;
+    ms.recb = recb;
+    int k = 0;
+    for (int m = 0; m < N; m++)
+      if (m != n) ms.other[k++] = m;
+    std::stable_sort(ms.other, ms.other + (N - 1), [&](int a, int b) { return X->dims[a] < X->dims[b]; });
+    // select this rank's nonzeros of mode n (stable)
+    DevBuf flag, incl, sel;
+    int64_t ns = 0;
+    CSTF_TRY(flag.alloc((size_t)nout * 4));
+    CSTF_TRY(incl.alloc((size_t)nout * 4));
+    if (nout) {
+      k_flag_range<<<grid_for(nout), kThreads, 0, st>>>(lab_idx[n].as<int32_t>(), nout, (int32_t)(rk * B),
+                                                        (int32_t)((rk + 1) * B), flag.as<uint32_t>());
+      CSTF_LAUNCHED();
+      size_t tb = 0;
+      CSTF_CUDA(cub::DeviceScan::InclusiveSum(nullptr, tb, flag.as<uint32_t>(), incl.as<uint32_t>(), nout, st));
+      CSTF_TRY(tmp.ensure(tb));
+      CSTF_CUDA(cub::DeviceScan::InclusiveSum(tmp.p, tb, flag.as<uint32_t>(), incl.as<uint32_t>(), nout, st));
+      count_launch();
+      uint32_t last = 0;
+      CSTF_CUDA(cudaMemcpyAsync(&last, incl.as<uint32_t>() + nout - 1, 4, cudaMemcpyDeviceToHost, st));
+      CSTF_CUDA(cudaStreamSynchronize(st));
+      ns = last;
+    }
+    CSTF_TRY(sel.alloc((size_t)ns * 4));
+    if (nout) {
+      k_scatter_sel<<<grid_for(nout), kThreads, 0, st>>>(flag.as<uint32_t>(), incl.as<uint32_t>(), nout,
+                                                         sel.as<uint32_t>());
+      CSTF_LAUNCHED();
+    }
+    // gathered keys: local row, then the other modes' internal labels by increasing length
+    DevBuf kk[8], vv;
+    for (int q = 0; q < N; q++) CSTF_TRY(kk[q].alloc((size_t)ns * 4));
+    CSTF_TRY(vv.alloc((size_t)ns * 8));
+    if (ns) {
+      k_gather_shift<<<grid_for(ns), kThreads, 0, st>>>(lab_idx[n].as<int32_t>(), sel.as<uint32_t>(), ns,
+                                                        (int32_t)(rk * B), kk[0].as<int32_t>());
+      CSTF_LAUNCHED();
+      for (int q = 0; q < N - 1; q++) {
+        k_gather_shift<<<grid_for(ns), kThreads, 0, st>>>(lab_idx[ms.other[q]].as<int32_t>(), sel.as<uint32_t>(), ns, 0,
+                                                          kk[q + 1].as<int32_t>());
+        CSTF_LAUNCHED();
+      }
+      k_gather<double><<<grid_for(ns), kThreads, 0, st>>>(c_vals.as<double>(), sel.as<uint32_t>(), ns,
+                                                          vv.as<double>());
+      CSTF_LAUNCHED();
+    }
+    const int32_t* keys[8];
+    int64_t kd[8];
+    keys[0] = kk[0].as<int32_t>();
+    kd[0] = B;
+    for (int q = 0; q < N - 1; q++) {
+      keys[q + 1] = kk[q + 1].as<int32_t>();
+      kd[q + 1] = (int64_t)P * X->rows_per_rank[ms.other[q]];
+    }
+    DevBuf pm;
+    CSTF_TRY(lsd_sort(keys, kd, N, ns, pm, tmp, st));
+    CSTF_TRY(build_rowptr(kk[0].as<int32_t>(), ns, B, ms.rowptr, tmp, st));
+    ms.nnz = ns;
+    CSTF_TRY(ms.rec.alloc((size_t)ns * recb));
+    RecArgs ra;
+    ra.nslots = N - 1;
+    ra.recb = recb;
+    for (int q = 0; q < N - 1; q++) ra.idx[q] = kk[q + 1].as<int32_t>();
+    if (ns) {
+      k_make_records<<<grid_for(ns), kThreads, 0, st>>>(ra, vv.as<double>(), pm.as<uint32_t>(), ns, ms.rec.as<char>());
+      CSTF_LAUNCHED();
+    }
+    CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  return CSTF_OK;
+}
 
 cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const double* host_vals,
                         int64_t n, cudaStream_t st) {
@@ -402,6 +549,7 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     X->normX2 = hv[0];
     memcpy(&X->hash, &hv[1], 8);
   }
+  if (X->nranks > 1) return build_partitioned(X, c_idx, c_vals, nout, tmp, st);
   // ---- 6. per-mode copies: sorted by (i_n, other modes by increasing length), AoS records
   const int recb = record_bytes(N);
   for (int n_ = 0; n_ < N; n_++) {

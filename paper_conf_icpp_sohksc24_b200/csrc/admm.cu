@@ -233,24 +233,41 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
   }
 }
 
-// G[a][b] (full R x R, raw) from the per-CTA tile partials of k_admm_dmma<RP, true>.
-// Element e = lane*2 + i of pair (xa, xb) is G[8 xa + lane/4][8 xb + 2 (lane%4) + i].
-__global__ void k_gram_from_parts(const double* __restrict__ gpart, int nblocks, int NT, int R,
-                                  double* __restrict__ G) {
-  const int NP = NT * (NT + 1) / 2;
-  for (int x = blockIdx.x * blockDim.x + threadIdx.x; x < NP * 64; x += gridDim.x * blockDim.x) {
-    const int p = x / 64, e = x % 64, lane = e / 2, i = e % 2;
-    int xa = 0, rem = p;
-    while (rem >= NT - xa) { rem -= NT - xa; xa++; }
-    const int xb = xa + rem;
-    const int r = 8 * xa + lane / 4, c = 8 * xb + 2 * (lane % 4) + i;
-    if (r >= R || c >= R) continue;
-    if (xa == xb && r > c) continue;      // diagonal tile: upper triangle, mirrored
-    double s = 0.0;
-    for (int b = 0; b < nblocks; b++) s += gpart[(size_t)b * NP * 64 + x];
-    G[r * R + c] = s;
-    G[c * R + r] = s;
+// Fixed-order reduction over CTAs: thread t sums parts t, t + 256, ... in order,
+// then a fixed tree over the 256 threads (deterministic for a given grid).
+__device__ __forceinline__ double block_sum_fixed(const double* __restrict__ src, int nparts, size_t stride) {
+  __shared__ double red[256];
+  double s = 0.0;
+  for (int b = threadIdx.x; b < nparts; b += 256) s += src[(size_t)b * stride];
+  red[threadIdx.x] = s;
+  __syncthreads();
+  for (int k = 128; k > 0; k >>= 1) {
+    if (threadIdx.x < k) red[threadIdx.x] += red[threadIdx.x + k];
+    __syncthreads();
   }
+  const double r = red[0];
+  __syncthreads();
+  return r;
+}
+
+// G[a][b] (full R x R, raw) from the per-CTA tile partials of k_admm_dmma<RP, true>;
+// one 256-thread CTA per partial element.  Element e = lane*2 + i of pair (xa, xb)
+// is G[8 xa + lane/4][8 xb + 2 (lane%4) + i].
+__global__ void __launch_bounds__(256) k_gram_from_parts(const double* __restrict__ gpart, int nblocks, int NT,
+                                                         int R, double* __restrict__ G) {
+  const int NP = NT * (NT + 1) / 2;
+  const int x = blockIdx.x;
+  const double s = block_sum_fixed(gpart + x, nblocks, (size_t)NP * 64);
+  if (threadIdx.x != 0) return;
+  const int p = x / 64, e = x % 64, lane = e / 2, i = e % 2;
+  int xa = 0, rem = p;
+  while (rem >= NT - xa) { rem -= NT - xa; xa++; }
+  const int xb = xa + rem;
+  const int r = 8 * xa + lane / 4, c = 8 * xb + 2 * (lane % 4) + i;
+  if (r >= R || c >= R) return;
+  if (xa == xb && r > c) return;      // diagonal tile: upper triangle, mirrored
+  G[r * R + c] = s;
+  G[c * R + r] = s;
 }
 
 // Generic form for any R <= 128: one CTA row at a time, thread = column.
@@ -308,15 +325,13 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
   }
 }
 
-// sums[j0 + j][w] = sum over CTAs (fixed order) of slots[j][cta][w]
-__global__ void k_admm_sum(const double* __restrict__ slots, int nblocks, int kiters, int from, int j0,
-                           double* __restrict__ sums) {
-  for (int x = threadIdx.x + from * 4; x < kiters * 4; x += blockDim.x) {
-    const int j = x >> 2, w = x & 3;
-    double s = 0.0;
-    for (int b = 0; b < nblocks; b++) s += slots[((size_t)j * nblocks + b) * 4 + w];
-    sums[(size_t)(j0 + j) * 4 + w] = s;
-  }
+// sums[j0 + j][w] = fixed-order sum over CTAs of slots[j][cta][w]; one CTA per (j, w)
+__global__ void __launch_bounds__(256) k_admm_sum(const double* __restrict__ slots, int nblocks, int from, int j0,
+                                                  double* __restrict__ sums) {
+  const int x = from * 4 + blockIdx.x;
+  const int j = x >> 2, w = x & 3;
+  const double s = block_sum_fixed(slots + (size_t)j * nblocks * 4 + w, nblocks, 4);
+  if (threadIdx.x == 0) sums[(size_t)(j0 + j) * 4 + w] = s;
 }
 
 // Stop decision over iterations [j0, j0 + k): first j with r < tol nH and s < tol nU (D3),
@@ -492,12 +507,15 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
     }
     int grid = 0;
     CSTF_TRY(launch_kernel(k, grid, gram_now, st));
-    k_admm_sum<<<1, 64, 0, st>>>(k.slots, grid, kk, k.sums_from, j0, w.sums.as<double>());
-    CSTF_LAUNCHED();
-    nl += 2;
+    if (kk > k.sums_from) {
+      k_admm_sum<<<(kk - k.sums_from) * 4, 256, 0, st>>>(k.slots, grid, k.sums_from, j0, w.sums.as<double>());
+      CSTF_LAUNCHED();
+      nl++;
+    }
+    nl++;
     if (gram_now) {
       const int NT = ((R + 7) & ~7) / 8;
-      k_gram_from_parts<<<(NT * (NT + 1) / 2 * 64 + 127) / 128, 128, 0, st>>>(w.gpart.as<double>(), grid, NT, R, A.G);
+      k_gram_from_parts<<<NT * (NT + 1) / 2 * 64, 256, 0, st>>>(w.gpart.as<double>(), grid, NT, R, A.G);
       CSTF_LAUNCHED();
       nl++;
     }

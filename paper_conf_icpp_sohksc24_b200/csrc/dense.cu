@@ -164,9 +164,10 @@ __global__ void k_fill(double* __restrict__ d, int64_t n, double v) {
 }
 
 // One CTA.  S (from d_S or Hadamard of the Grams except `skip`, increasing k),
-// rho = tr(S)/R (or rho_in > 0), Cholesky-Banachiewicz of S + rho I in shared
-// memory (same summation order as Alg. 2's textbook form, no FMA contraction),
-// L^-1 by column-parallel forward substitution, Inv = L^-T L^-1.
+// rho = tr(S)/R (or rho_in > 0), right-looking Cholesky of S + rho I in shared
+// memory, L^-1 by forward substitution on all columns at once, Inv = L^-T L^-1
+// (pre-inversion, Sec. 4.3.2).  kappa(S + rho I) <= R + 1 (pin P5) keeps the
+// explicit inverse accurate.
 __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __restrict__ grams,
                                int N, int skip, int R, double rho_in, double* __restrict__ Linv,
                                double* __restrict__ Inv, double* __restrict__ scal, int* flag,
@@ -184,8 +185,9 @@ __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __
       colscale[R + r] = (ls > 0.0) ? 1.0 / ls : 0.0;
     }
   }
-  extern __shared__ double L[];  // [R][R]: A, then L in the lower triangle
+  extern __shared__ double L[];  // [R][R]: A, then L in the lower triangle; then [R][R] L^-1 if it fits
   __shared__ double s_rho;
+  if (R <= 64) Linv = L + R * R;   // shared-memory copy of L^-1 (latency-bound loops below)
   __shared__ int s_bad;
   const int RR = R * R;
   for (int e = threadIdx.x; e < RR; e += blockDim.x) {
@@ -220,33 +222,43 @@ __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __
   const double rho = s_rho;
   for (int a = threadIdx.x; a < R; a += blockDim.x) L[a * R + a] = __dadd_rn(L[a * R + a], rho);
   __syncthreads();
+  // right-looking Cholesky: step j scales column j and updates the trailing
+  // lower triangle in parallel (two barriers per step)
   for (int j = 0; j < R; j++) {
     if (threadIdx.x == 0) {
-      double s = L[j * R + j];
-      for (int k = 0; k < j; k++) s = __dsub_rn(s, __dmul_rn(L[j * R + k], L[j * R + k]));
-      if (!(s > 0.0)) { s_bad = 1; s = 1.0; }
-      L[j * R + j] = sqrt(s);
+      const double s = L[j * R + j];
+      if (!(s > 0.0)) s_bad = 1;
+      L[j * R + j] = sqrt(s > 0.0 ? s : 1.0);
     }
     __syncthreads();
     const double d = L[j * R + j];
-    for (int i = j + 1 + threadIdx.x; i < R; i += blockDim.x) {
-      double s = L[i * R + j];
-      for (int k = 0; k < j; k++) s = __dsub_rn(s, __dmul_rn(L[i * R + k], L[j * R + k]));
-      L[i * R + j] = s / d;
+    for (int i = j + 1 + threadIdx.x; i < R; i += blockDim.x) L[i * R + j] = L[i * R + j] / d;
+    __syncthreads();
+    const int m = R - j - 1;                      // trailing block (j+1..R-1)^2, lower part
+    for (int e = threadIdx.x; e < m * m; e += blockDim.x) {
+      const int i = j + 1 + e / m, k = j + 1 + e % m;
+      if (k <= i) L[i * R + k] = fma(-L[i * R + j], L[k * R + j], L[i * R + k]);
     }
     __syncthreads();
   }
-  // Linv column c: forward substitution of L y = e_c (global scratch, R x R)
-  for (int c = threadIdx.x; c < R; c += blockDim.x) {
-    for (int a = 0; a < c; a++) Linv[a * R + c] = 0.0;
-    Linv[c * R + c] = 1.0 / L[c * R + c];
-    for (int a = c + 1; a < R; a++) {
-      double s = 0.0;
-      for (int k = c; k < a; k++) s = fma(L[a * R + k], Linv[k * R + c], s);
-      Linv[a * R + c] = -s / L[a * R + a];
-    }
+  // L^-1 by forward substitution on all columns at once: step a fixes row a
+  // of L^-1, then eliminates it from the rows below
+  for (int e = threadIdx.x; e < R * R; e += blockDim.x) {
+    const int i = e / R, c = e % R;
+    Linv[e] = (i == c) ? 1.0 : 0.0;
   }
   __syncthreads();
+  for (int a = 0; a < R; a++) {
+    const double inv_d = 1.0 / L[a * R + a];
+    for (int c = threadIdx.x; c <= a; c += blockDim.x) Linv[a * R + c] *= inv_d;
+    __syncthreads();
+    const int m = R - a - 1;
+    for (int e = threadIdx.x; e < m * (a + 1); e += blockDim.x) {
+      const int i = a + 1 + e / (a + 1), c = e % (a + 1);
+      Linv[i * R + c] = fma(-L[i * R + a], Linv[a * R + c], Linv[i * R + c]);
+    }
+    __syncthreads();
+  }
   // Inv[a][b] = sum_{k >= max(a,b)} Linv[k][a] Linv[k][b]   (computed for a <= b, mirrored)
   for (int e = threadIdx.x; e < RR; e += blockDim.x) {
     const int a = e / R, b = e % R;
@@ -391,7 +403,7 @@ cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int sk
                          cudaStream_t st, const double* d_lam, double* d_colscale) {
   Workspace& w = ws();
   CSTF_TRY(w.linv.ensure((size_t)R * R * 8));
-  const size_t smem = (size_t)R * R * 8;
+  const size_t smem = (size_t)R * R * 8 * (R <= 64 ? 2 : 1);
   static bool attr_set = false;
   if (!attr_set) {
     CSTF_CUDA(cudaFuncSetAttribute(k_chol_inverse, cudaFuncAttributeMaxDynamicSharedMemorySize, 128 * 1024));

@@ -277,7 +277,10 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
 }
 
 // Add the carries of every row that continues across chunks, in chunk order.
-__global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks,
+// The run of carry chunks of row h ends at the chunk holding h's last nonzero
+// (known from rowptr), so the loop has a known trip count and its loads pipeline.
+__global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks, const int64_t* __restrict__ rowptr,
+                              int64_t chunk, const int64_t* __restrict__ wstart,
                               const double* __restrict__ carry, int R, double* __restrict__ M) {
   const int lane = threadIdx.x & 31;
   const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -285,10 +288,30 @@ __global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks,
   for (int64_t c = warp0; c < nchunks; c += nwarps) {
     const int32_t h = cont[c];
     if (h < 0 || (c > 0 && cont[c - 1] == h)) continue;
+    const int64_t plast = rowptr[h + 1] - 1;           // last nonzero of row h
+    int64_t cend;                                      // chunk holding plast
+    if (!wstart) {
+      cend = plast / chunk;
+    } else {
+      int64_t lo = c, hi = nchunks - 1;                // last chunk with wstart <= plast
+      while (lo < hi) {
+        const int64_t mid = (lo + hi + 1) >> 1;
+        if (wstart[mid] <= plast) lo = mid; else hi = mid - 1;
+      }
+      cend = lo;
+    }
     for (int col = lane; col < R; col += 32) {
-      double s = 0.0;
-      for (int64_t cc = c; cc < nchunks && cont[cc] == h; cc++) s += carry[cc * R + col];
-      M[(int64_t)h * R + col] += s;
+      // four interleaved partial sums (fixed combination order) keep 16 loads in flight
+      double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
+      int64_t cc = c;
+      for (; cc + 3 <= cend; cc += 4) {
+        s0 += carry[cc * R + col];
+        s1 += carry[(cc + 1) * R + col];
+        s2 += carry[(cc + 2) * R + col];
+        s3 += carry[(cc + 3) * R + col];
+      }
+      for (; cc <= cend; cc++) s0 += carry[cc * R + col];
+      M[(int64_t)h * R + col] += (s0 + s1) + (s2 + s3);
     }
   }
 }
@@ -479,7 +502,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   nl++;
   if (nchunks > 1) {
     const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);
-    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.carry, R, out);
+    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, a.carry, R, out);
     CSTF_LAUNCHED();
     nl++;
   }

@@ -37,6 +37,8 @@ bool rank_ok(int R) { return R >= 1 && R <= 128; }
 struct DriverWs {
   DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8];
   double* host_small = nullptr;  // pinned: fit, flags
+  cudaStream_t side = nullptr;   // the R x R step of a mode overlaps its MTTKRP
+  cudaEvent_t fork = nullptr, join = nullptr;
 };
 DriverWs& dws() {
   static thread_local DriverWs w[64];
@@ -44,6 +46,11 @@ DriverWs& dws() {
   cudaGetDevice(&dev);
   DriverWs& r = w[dev & 63];
   if (!r.host_small) cudaMallocHost(&r.host_small, 64 * sizeof(double));
+  if (!r.side) {
+    cudaStreamCreateWithFlags(&r.side, cudaStreamNonBlocking);
+    cudaEventCreateWithFlags(&r.fork, cudaEventDisableTiming);
+    cudaEventCreateWithFlags(&r.join, cudaEventDisableTiming);
+  }
   return r;
 }
 
@@ -184,14 +191,17 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       const int64_t I = Iloc[n];
       double* Hn = fac[n] + off[n];     // this rank's rows of the raw factor
       double* Gn = G + (size_t)n * R * R;
-      // a1 + a3 + a4: S = *_{k!=n} G^(k), rho, Cholesky, Inv   (GRAM phase)
-      tm.begin(n, CSTF_PHASE_GRAM);
-      CSTF_TRY(chol_inverse(nullptr, G, N, n, R, o->admm.rho, w.inv.as<double>(), w.scal.as<double>(), flag, st,
-                            lam, colscale));
-      tm.end(n, CSTF_PHASE_GRAM);
-      // a2: MTTKRP of the raw factors
+      // a1 + a3 + a4 (S, rho, Cholesky, Inv: one CTA) run on a side stream,
+      // concurrently with a2 (MTTKRP) which does not depend on them
+      CSTF_CUDA(cudaEventRecord(w.fork, st));
+      CSTF_CUDA(cudaStreamWaitEvent(w.side, w.fork, 0));
+      CSTF_TRY(chol_inverse(nullptr, G, N, n, R, o->admm.rho, w.inv.as<double>(), w.scal.as<double>(), flag,
+                            w.side, lam, colscale));
+      CSTF_CUDA(cudaEventRecord(w.join, w.side));
+      // a2: MTTKRP of the raw factors (MTTKRP phase = both, overlapped)
       tm.begin(n, CSTF_PHASE_MTTKRP);
       CSTF_TRY(mttkrp(X, n, R, fac.data(), M, st, nullptr));
+      CSTF_CUDA(cudaStreamWaitEvent(st, w.join, 0));
       tm.end(n, CSTF_PHASE_MTTKRP);
       // a5: ADMM on M diag(mscale); warm start H_raw (D4) or the normalised H (literal)
       tm.begin(n, CSTF_PHASE_UPDATE);

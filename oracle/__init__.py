@@ -21,7 +21,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 OK, EINVAL, ENOMEM, NOT_SPD, NUMERIC = 0, 1, 3, 6, 7
-PROX_NONNEG, PROX_IDENTITY = 0, 1
+PROX_NONNEG, PROX_IDENTITY, PROX_L1, PROX_NONNEG_L1 = 0, 1, 2, 3
 WARM_SCALED, WARM_NORMALIZED = 0, 1
 
 
@@ -55,11 +55,11 @@ def _get():
         L.oracle_gram.argtypes = [i64, i32, p, p]
         L.oracle_hadamard_except.argtypes = [i32, i32, p, i32, p]
         L.oracle_cholesky.argtypes = [i32, p, p]
-        L.oracle_admm.argtypes = [i64, i32, p, p, p, p, d, i32, d, i32, p, p]
+        L.oracle_admm.argtypes = [i64, i32, p, p, p, p, d, i32, d, i32, d, p, p]
         L.oracle_normalize.argtypes = [i64, i32, p, p]
         L.oracle_fit.restype = d
         L.oracle_fit.argtypes = [i32, i32, d, i64, p, p, p, p]
-        L.oracle_factorize.argtypes = [i32, p, i64, p, p, d, i32, i32, d, d, i32, d, i32, i32, i32,
+        L.oracle_factorize.argtypes = [i32, p, i64, p, p, d, i32, i32, d, d, i32, d, i32, i32, i32, d,
                                        p, p, p, p, p, p, p]
         _lib = L
     return _lib
@@ -176,7 +176,7 @@ def cholesky(A) -> np.ndarray:
     return L
 
 
-def admm(M, S, H, U, tol=0.0, max_iter=10, rho=0.0, prox=PROX_NONNEG, trace=False):
+def admm(M, S, H, U, tol=0.0, max_iter=10, rho=0.0, prox=PROX_NONNEG, trace=False, alpha=0.0):
     """O7: Alg. 2 (L550-580). Returns (H, U, stats dict[, trace array])."""
     M = _c64(M); S = _c64(S)
     H = np.array(H, dtype=np.float64, copy=True, order="C")
@@ -185,7 +185,7 @@ def admm(M, S, H, U, tol=0.0, max_iter=10, rho=0.0, prox=PROX_NONNEG, trace=Fals
     stats = np.zeros(6)
     tr = np.zeros((max_iter, 4)) if trace else None
     st = _get().oracle_admm(I, R, M.ctypes.data, S.ctypes.data, H.ctypes.data, U.ctypes.data,
-                            float(tol), int(max_iter), float(rho), int(prox), stats.ctypes.data,
+                            float(tol), int(max_iter), float(rho), int(prox), float(alpha), stats.ctypes.data,
                             tr.ctypes.data if trace else None)
     if st:
         raise OracleError(st, "admm")
@@ -215,7 +215,7 @@ def fit(normX2, M_last, H_last, lam, grams) -> float:
 
 
 def factorize(X: Tensor, factors, outer_iters=10, tol=1e-2, max_iter=10, rho=0.0,
-              warm=WARM_SCALED, normalize_init=True, prox=PROX_NONNEG, fit_tol=0.0):
+              warm=WARM_SCALED, normalize_init=True, prox=PROX_NONNEG, fit_tol=0.0, alpha=0.0):
     """O9/O11: Alg. 1 (L476-506) with readings D4, D6, D11, D13.
 
     Returns dict(factors, lam (N x R), fit[outer_done], iters[outer_done x N], phase_ms[4],
@@ -233,7 +233,7 @@ def factorize(X: Tensor, factors, outer_iters=10, tol=1e-2, max_iter=10, rho=0.0
     st = _get().oracle_factorize(N, dims_a.ctypes.data, X.nnz, _ptrs(X.idx), X.vals.ctypes.data,
                                  float(X.normX2), R, int(outer_iters), float(fit_tol), float(tol),
                                  int(max_iter), float(rho), int(warm), int(bool(normalize_init)),
-                                 int(prox), _ptrs(H), lam.ctypes.data, fits.ctypes.data,
+                                 int(prox), float(alpha), _ptrs(H), lam.ctypes.data, fits.ctypes.data,
                                  iters.ctypes.data, ctypes.byref(done), phase.ctypes.data,
                                  trace.ctypes.data)
     if st:

@@ -42,6 +42,18 @@
 
 #define PROX_NONNEG 0   /* indicator of R_+ : max(0, x), L835-839 */
 #define PROX_IDENTITY 1 /* unconstrained (pin P10: reduces to CP-ALS, L360-368) */
+#define PROX_L1 2       /* r(H) = alpha ||H||_1: soft threshold at alpha/rho (L540-541, L615-619) */
+#define PROX_NONNEG_L1 3 /* r(H) = alpha ||H||_1 + indicator(R_+): max(0, x - alpha/rho) */
+
+/* Alg. 2 l.7: argmin_h r(h) + rho/2 (h - x)^2 for the element-wise regularisers above */
+static double prox_apply(int prox, double x, double tau) {
+  switch (prox) {
+    case PROX_IDENTITY: return x;
+    case PROX_L1: return x > tau ? x - tau : (x < -tau ? x + tau : 0.0);
+    case PROX_NONNEG_L1: return x > tau ? x - tau : 0.0;
+    default: return x > 0.0 ? x : 0.0;
+  }
+}
 
 static double now_ms(void) {
   struct timespec ts; clock_gettime(CLOCK_MONOTONIC, &ts);
@@ -271,14 +283,15 @@ int oracle_cholesky(int R, const double* A, double* L) {
  *   H0 <- H                                   (l.5, reading D2)
  *   H~ <- (L L^T)^{-1} (M + rho (H + U))      (l.6, row-major reading D1:
  *                                              forward then back substitution per row)
- *   H  <- prox(H~ - U)                        (l.7; nonneg: x > 0 ? x : +0.0, D15)
+ *   H  <- prox(H~ - U)                        (l.7; nonneg: x > 0 ? x : +0.0, D15;
+ *                                              L1 variants threshold at alpha/rho)
  *   U  <- U + H - H~                          (l.8)
  * until ||H - H~||^2 < eps ||H||^2 and ||H - H0||^2 < eps ||U||^2 (l.9, reading D3:
  *   squared norms of the UPDATED H, U, strict <, no division, at least one pass).
  * stats = {iters, rho, r, s, nH, nU} of the last pass; trace (optional) gets the
  * four sums of every pass [max_iter][4]. */
 int oracle_admm(int64_t I, int R, const double* M, const double* S, double* H, double* U,
-                double tol, int max_iter, double rho_in, int prox, double* stats, double* trace) {
+                double tol, int max_iter, double rho_in, int prox, double alpha, double* stats, double* trace) {
   if (R < 1 || max_iter < 1 || I < 0) return ORC_EINVAL;
   double rho = 0.0;
   if (rho_in > 0.0) rho = rho_in;
@@ -288,6 +301,7 @@ int oracle_admm(int64_t I, int R, const double* M, const double* S, double* H, d
     rho = tr / R;
   }
   if (!(rho > 0.0)) return ORC_NOT_SPD;
+  const double tau = alpha / rho;
   double* A = (double*)malloc((size_t)R * R * sizeof(double));
   double* L = (double*)malloc((size_t)R * R * sizeof(double));
   for (int e = 0; e < R * R; e++) A[e] = S[e];
@@ -322,7 +336,7 @@ int oracle_admm(int64_t I, int R, const double* M, const double* S, double* H, d
         }
         for (int c = 0; c < R; c++) {
           double d = x[c] - u[c];
-          double hn = (prox == PROX_IDENTITY) ? d : (d > 0.0 ? d : 0.0);
+          double hn = prox_apply(prox, d, tau);
           double un = u[c] + hn - x[c];
           double e1 = hn - x[c], e2 = hn - h0[c];
           pr = pr + e1 * e1; ps = ps + e2 * e2; ph = ph + hn * hn; pu = pu + un * un;
@@ -417,7 +431,7 @@ double oracle_fit(int N, int R, double normX2, int64_t I_last, const double* M_l
 int oracle_factorize(int N, const int64_t* dims, int64_t nnz, const int32_t* const* cidx,
                      const double* cvals, double normX2, int R, int outer_iters, double fit_tol,
                      double tol, int max_iter, double rho_in, int warm, int normalize_init, int prox,
-                     double* const* H, double* lam_all, double* fit_out, int* iters_out,
+                     double alpha, double* const* H, double* lam_all, double* fit_out, int* iters_out,
                      int* outer_done, double* phase_ms, double* trace_out) {
   if (N < 2 || N > 8 || R < 1 || R > 128 || outer_iters < 1 || max_iter < 1) return ORC_EINVAL;
   int st = ORC_OK;
@@ -455,7 +469,7 @@ int oracle_factorize(int N, const int64_t* dims, int64_t nnz, const int32_t* con
       }
       double stats[6];
       double* tr = trace_out ? trace_out + ((size_t)t * N + n) * (size_t)max_iter * 4 : NULL;
-      st = oracle_admm(dims[n], R, M, S, H[n], U[n], tol, max_iter, rho_in, prox, stats, tr);
+      st = oracle_admm(dims[n], R, M, S, H[n], U[n], tol, max_iter, rho_in, prox, alpha, stats, tr);
       if (st) break;
       if (iters_out) iters_out[t * N + n] = (int)stats[0];
       double t3 = now_ms();

@@ -24,7 +24,7 @@ c_void_p, c_int, c_int64, c_double = ctypes.c_void_p, ctypes.c_int, ctypes.c_int
 # status codes
 CSTF_OK, CSTF_ERR_INVALID_ARG, CSTF_ERR_UNSUPPORTED, CSTF_ERR_OUT_OF_MEMORY = 0, 1, 2, 3
 CSTF_ERR_CUDA, CSTF_ERR_NCCL, CSTF_ERR_NOT_SPD, CSTF_ERR_NUMERIC = 4, 5, 6, 7
-CSTF_PROX_NONNEG, CSTF_PROX_IDENTITY = 0, 1
+CSTF_PROX_NONNEG, CSTF_PROX_IDENTITY, CSTF_PROX_L1, CSTF_PROX_NONNEG_L1 = 0, 1, 2, 3
 CSTF_ADMM_AUTO, CSTF_ADMM_STREAMING, CSTF_ADMM_RESIDENT = 0, 1, 2
 CSTF_WARM_SCALED, CSTF_WARM_NORMALIZED = 0, 1
 PHASES = ("GRAM", "MTTKRP", "UPDATE", "NORMALIZE", "COMM")
@@ -40,7 +40,7 @@ class CstfError(RuntimeError):
 
 class AdmmOpts(ctypes.Structure):
     _fields_ = [("tol", c_double), ("max_iter", c_int), ("rho", c_double), ("prox", c_int),
-                ("variant", c_int)]
+                ("variant", c_int), ("alpha", c_double)]
 
 
 class AdmmStats(ctypes.Structure):
@@ -306,14 +306,15 @@ def cstf_normalize(H, lam, G=None, comm=None, stream=None):
     return H, lam
 
 
-def admm_opts(tol=0.0, max_iter=10, rho=0.0, prox=CSTF_PROX_NONNEG, variant=CSTF_ADMM_AUTO) -> AdmmOpts:
-    return AdmmOpts(float(tol), int(max_iter), float(rho), int(prox), int(variant))
+def admm_opts(tol=0.0, max_iter=10, rho=0.0, prox=CSTF_PROX_NONNEG, variant=CSTF_ADMM_AUTO,
+              alpha=0.0) -> AdmmOpts:
+    return AdmmOpts(float(tol), int(max_iter), float(rho), int(prox), int(variant), float(alpha))
 
 
 def cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, rho=0.0, prox=CSTF_PROX_NONNEG,
-                     variant=CSTF_ADMM_AUTO, comm=None, stream=None) -> dict:
+                     variant=CSTF_ADMM_AUTO, comm=None, stream=None, alpha=0.0) -> dict:
     I, R = H.shape
-    o = admm_opts(tol, max_iter, rho, prox, variant)
+    o = admm_opts(tol, max_iter, rho, prox, variant, alpha)
     st = AdmmStats()
     _check(_lib.cstf_admm_update(_dptr(M), _dptr(S), _dptr(H), _dptr(U), I, R, ctypes.byref(o), _comm(comm),
                                  ctypes.byref(st), _stream(stream)), "cstf_admm_update")
@@ -321,8 +322,9 @@ def cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, rho=0.0, prox=CSTF_PROX_N
 
 
 def make_opts(R, outer_iters=10, fit_tol=0.0, tol=1e-2, max_iter=10, rho=0.0, prox=CSTF_PROX_NONNEG,
-              variant=CSTF_ADMM_AUTO, warm=CSTF_WARM_SCALED, normalize_init=True, timing=False) -> Opts:
-    return Opts(int(R), int(outer_iters), float(fit_tol), admm_opts(tol, max_iter, rho, prox, variant),
+              variant=CSTF_ADMM_AUTO, warm=CSTF_WARM_SCALED, normalize_init=True, timing=False,
+              alpha=0.0) -> Opts:
+    return Opts(int(R), int(outer_iters), float(fit_tol), admm_opts(tol, max_iter, rho, prox, variant, alpha),
                 int(warm), int(bool(normalize_init)), int(bool(timing)))
 
 

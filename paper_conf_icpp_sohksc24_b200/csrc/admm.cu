@@ -49,11 +49,22 @@ struct KArgs {
   const double* scal;      // [0] = rho
   const int* flag;         // skip all work if a previous step failed
   int prox;
+  double alpha;            // L1 weight; threshold tau = alpha / rho
   int kiters;
   int sums_from;           // first local pass whose residual sums are formed
   double* slots;           // [kiters][gridDim][4]
   double* gpart;           // optional: per-CTA Gram partials [grid][NT(NT+1)/2][64]
 };
+
+// Alg. 2 l.7: argmin_h r(h) + rho/2 (h - x)^2 for the element-wise regularisers
+__device__ __forceinline__ double prox_apply(int prox, double x, double tau) {
+  switch (prox) {
+    case CSTF_PROX_IDENTITY: return x;
+    case CSTF_PROX_L1: return x > tau ? x - tau : (x < -tau ? x + tau : 0.0);
+    case CSTF_PROX_NONNEG_L1: return x > tau ? x - tau : 0.0;
+    default: return x > 0.0 ? x : 0.0;
+  }
+}
 
 __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b) {
   asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
@@ -77,6 +88,7 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
   const int R = a.R;
   const bool skip = *a.flag != 0;   // an earlier step failed: write zero sums, touch nothing
   const double rho = a.scal[0];
+  const double tau = a.alpha / rho;
   const int kiters = a.kiters;
   for (int x = tid; x < nsl * 4 * kThreads; x += kThreads) sacc[x] = 0.0;
   if (GRAM)
@@ -152,7 +164,7 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
           for (int i = 0; i < 2; i++) {
             const double ht = d[t][i];
             const double x = ht - u[t][i];
-            const double hn = (a.prox == CSTF_PROX_IDENTITY) ? x : (x > 0.0 ? x : 0.0);
+            const double hn = prox_apply(a.prox, x, tau);
             const double un = (u[t][i] + hn) - ht;
             const double e1 = hn - ht, e2 = hn - h[t][i];
             pr = fma(e1, e1, pr); ps = fma(e2, e2, ps); ph = fma(hn, hn, ph); pu = fma(un, un, pu);
@@ -168,7 +180,7 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
           for (int i = 0; i < 2; i++) {
             const double ht = d[t][i];
             const double x = ht - u[t][i];
-            const double hn = (a.prox == CSTF_PROX_IDENTITY) ? x : (x > 0.0 ? x : 0.0);
+            const double hn = prox_apply(a.prox, x, tau);
             u[t][i] = (u[t][i] + hn) - ht;
             h[t][i] = hn;
           }
@@ -280,6 +292,7 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
   const int R = a.R;
   const bool skip = *a.flag != 0;
   const double rho = a.scal[0];
+  const double tau = a.alpha / rho;
   const int kiters = a.kiters;
   for (int x = tid; x < R * R; x += blockDim.x) sinv[x] = a.inv[x];
   for (int x = tid; x < kiters * 4 * 128; x += blockDim.x) sacc[x] = 0.0;
@@ -300,7 +313,7 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
         for (int k = 0; k < R; k++) ht = fma(st[k], sinv[k * R + tid], ht);
       __syncthreads();
       const double x = ht - u;
-      const double hn = (a.prox == CSTF_PROX_IDENTITY) ? x : (x > 0.0 ? x : 0.0);
+      const double hn = prox_apply(a.prox, x, tau);
       const double un = (u + hn) - ht;
       const double e1 = hn - ht, e2 = hn - h;
       if (cok) {
@@ -475,6 +488,7 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
   k.scal = A.scal;
   k.flag = A.flag;
   k.prox = A.prox;
+  k.alpha = A.alpha;
   k.slots = w.slots.as<double>();
   k.gpart = nullptr;
   if (spec) {

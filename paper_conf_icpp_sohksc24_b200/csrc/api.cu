@@ -110,6 +110,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   const int R = o->R;
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
   if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
+  if (o->admm.prox < CSTF_PROX_NONNEG || o->admm.prox > CSTF_PROX_NONNEG_L1 || !(o->admm.alpha >= 0.0))
+    return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
   const bool dist = X->nranks > 1;
   if (comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
     return fail(CSTF_ERR_INVALID_ARG, "comm does not match the tensor's partition");
@@ -211,6 +213,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       a.hscale = (o->warm == CSTF_WARM_SCALED) ? nullptr : colscale + R;
       a.I = I; a.R = R; a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
       a.tol = o->admm.tol; a.max_iter = o->admm.max_iter; a.prox = o->admm.prox; a.variant = o->admm.variant;
+      a.alpha = o->admm.alpha;
       const bool fused = admm_can_fuse_gram(R, o->admm.tol);
       a.G = fused ? Gn : nullptr;      // a7 fused into the ADMM epilogue
       int iters = 0;
@@ -345,8 +348,8 @@ cstf_status cstf_admm_update(const double* d_M, const double* d_S, double* d_H, 
     return fail(CSTF_ERR_INVALID_ARG, "NULL argument or I < 0");
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
   if (opts->max_iter < 1 || opts->tol < 0.0) return fail(CSTF_ERR_INVALID_ARG, "max_iter < 1 or tol < 0");
-  if (opts->prox != CSTF_PROX_NONNEG && opts->prox != CSTF_PROX_IDENTITY)
-    return fail(CSTF_ERR_INVALID_ARG, "unknown prox");
+  if (opts->prox < CSTF_PROX_NONNEG || opts->prox > CSTF_PROX_NONNEG_L1 || !(opts->alpha >= 0.0))
+    return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
   cudaStream_t st = S(stream);
   DriverWs& w = dws();
   CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
@@ -359,6 +362,7 @@ cstf_status cstf_admm_update(const double* d_M, const double* d_S, double* d_H, 
   a.M = d_M; a.H = d_H; a.U = d_U; a.hscale = nullptr; a.I = I; a.R = R;
   a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
   a.tol = opts->tol; a.max_iter = opts->max_iter; a.prox = opts->prox; a.variant = opts->variant;
+  a.alpha = opts->alpha;
   cstf_admm_stats stats;
   CSTF_TRY(admm_run(a, comm, st, &stats, nullptr, nullptr));
   CSTF_TRY(check_flag(flag, st));

@@ -198,6 +198,7 @@ struct AdmmArgs {
   int max_iter;
   int prox;
   int variant;
+  double alpha = 0.0;    // L1 weight (prox 2/3)
 };
 cstf_status admm_run(const AdmmArgs& a, const cstf_comm* comm, cudaStream_t st,
                      cstf_admm_stats* stats, int* iters_out, int64_t* launches);

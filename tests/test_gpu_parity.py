@@ -339,3 +339,34 @@ def test_mttkrp_kblocked_with_empty_blocks(B, R):
         M = cu(np.full((dims[n], R), np.nan))
         B.cstf_mttkrp(X, n, Fd, M)
         assert normwise(host(M), oracle.mttkrp(ref, n, F)) <= TOL, n
+
+
+@pytest.mark.parametrize("prox", [2, 3])
+@pytest.mark.parametrize("R,variant", [(8, 0), (32, 0), (32, 1), (64, 0), (100, 0)])
+def test_admm_l1_prox(B, prox, R, variant):
+    """f3: L1 soft-threshold (and its non-negative form) in the fused kernel vs the oracle."""
+    M, S, H, U = admm_inputs(1500, R, 7 + R)
+    alpha = 0.2 * float(np.mean(np.diag(S)))
+    Hd, Ud = cu(H), cu(U)
+    st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=0.0, max_iter=10, prox=prox, alpha=alpha, variant=variant)
+    Hr, Ur, sr = oracle.admm(M, S, H, U, tol=0.0, max_iter=10, prox=prox, alpha=alpha)
+    assert normwise(host(Hd), Hr) <= TOL and normwise(host(Ud), Ur) <= TOL
+    got = host(Hd)
+    assert np.mean(got == 0.0) > 0.05                 # the threshold produces exact zeros
+    if prox == 2:
+        assert np.any(got < 0)
+
+
+def test_factorize_nonneg_l1(B):
+    c = datagen.CONFIGS["nell2"].scaled(40, nnz_factor=800)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, 16, c.seed)
+    ref = oracle.coalesce(c.dims, idx, vals)
+    orc = oracle.factorize(ref, start, outer_iters=5, tol=1e-2, max_iter=10, prox=oracle.PROX_NONNEG_L1, alpha=0.5)
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    F = [cu(f) for f in start]
+    lam = cu(np.zeros(16))
+    gpu = B.cstf_factorize(X, F, lam, B.make_opts(16, outer_iters=5, tol=1e-2, prox=3, alpha=0.5))
+    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
+    assert tie is None
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6

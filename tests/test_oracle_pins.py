@@ -398,3 +398,49 @@ def test_P11_thread_count_determinism():
         env = dict(os.environ, OMP_NUM_THREADS=th, PYTHONPATH=os.path.dirname(HERE))
         out.append(subprocess.check_output([sys.executable, "-c", code], env=env).strip())
     assert out[0] == out[1] == out[2]
+
+
+# --------------------------------------------------------------------- f3: L1 proximity operators
+def lasso_bruteforce(S, m, alpha, nonneg):
+    """min_h 1/2 h^T S h - m^T h + alpha ||h||_1 (h >= 0 if nonneg) by enumerating
+    sign patterns (each coordinate -, 0, +): on a fixed pattern the problem is an
+    equality-constrained quadratic with the linear term shifted by alpha*sign."""
+    from itertools import product
+    R = len(m)
+    best, best_h = np.inf, None
+    signs = (0, 1) if nonneg else (-1, 0, 1)
+    for pat in product(signs, repeat=R):
+        P = [i for i in range(R) if pat[i] != 0]
+        h = np.zeros(R)
+        if P:
+            sg = np.array([pat[i] for i in P], dtype=float)
+            h[P] = np.linalg.solve(S[np.ix_(P, P)], m[P] - alpha * sg)
+            if np.any(np.sign(h[P]) != sg):
+                continue
+        f = 0.5 * h @ S @ h - m @ h + alpha * np.abs(h).sum()
+        if f < best:
+            best, best_h = f, h
+    return best_h
+
+
+@pytest.mark.parametrize("prox,nonneg", [(oracle.PROX_L1, False), (oracle.PROX_NONNEG_L1, True)])
+@pytest.mark.parametrize("R", [2, 3])
+def test_f3_l1_prox_fixed_point_is_lasso(rng, prox, nonneg, R):
+    """ADMM with r = alpha ||.||_1 (+ R_+) converges to the brute-force (non-negative) lasso."""
+    S = make_S(rng, R)
+    I = 30
+    M = (rng.random((I, R)) - 0.4) * np.diag(S).mean()
+    alpha = 0.3 * np.diag(S).mean()
+    H, U, st = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), tol=0.0, max_iter=6000, prox=prox, alpha=alpha)
+    ref = np.array([lasso_bruteforce(S, M[i], alpha, nonneg) for i in range(I)])
+    assert np.any(ref == 0.0)
+    assert normwise(H, ref) <= 1e-9
+
+
+def test_f3_l1_with_zero_alpha_is_the_plain_operator(rng):
+    R, I = 5, 40
+    S = make_S(rng, R)
+    M = rng.random((I, R)) - 0.5
+    a = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), max_iter=20, prox=oracle.PROX_NONNEG_L1, alpha=0.0)
+    b = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), max_iter=20, prox=oracle.PROX_NONNEG)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])

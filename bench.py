@@ -45,6 +45,16 @@ def load_peaks():
         return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0}, "fallback (B200_PROFILING.md)"
 
 
+def measured_traffic(workload):
+    """DRAM bytes per launch of the dominant kernel from the committed ncu capture (or None)."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
+            t = json.load(f).get(workload)
+        return None if t is None else t["dram_read"] + t["dram_write"]
+    except Exception:
+        return None
+
+
 def env_rank():
     return int(os.environ.get("RANK", 0)), int(os.environ.get("WORLD_SIZE", 1)), int(os.environ.get("LOCAL_RANK", 0))
 
@@ -133,6 +143,37 @@ def run_reference(args, cfg):
     return 0
 
 
+def admm_ablation(B, cfg, R, stream, reps=5):
+    """SURVEY f2 / Fig. 4 analogue on this workload's mode shapes: one ADMM update
+    (10 inner iterations, eps = 0) per mode, streaming vs row-resident kernel."""
+    import torch
+    import oracle   # only to build a realistic S (Hadamard of Grams of normalised factors)
+    out = {}
+    for n, I in enumerate(cfg.dims):
+        Fs = [oracle.normalize(datagen.uniform(cfg.seed, 50 + k, 256 * R).reshape(256, R))[0]
+              for k in range(len(cfg.dims))]
+        S = torch.from_numpy(oracle.hadamard_except([oracle.gram(f) for f in Fs], n)).cuda()
+        M = torch.rand(I, R, dtype=torch.float64, device="cuda")
+        H0 = torch.rand(I, R, dtype=torch.float64, device="cuda")
+        res = {}
+        for name, var in (("streaming", B.CSTF_ADMM_STREAMING), ("resident", B.CSTF_ADMM_RESIDENT)):
+            H, U = H0.clone(), torch.zeros_like(H0)
+            B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=var)
+            ts = []
+            for _ in range(reps):
+                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=var)
+                b.record(stream)
+                torch.cuda.synchronize()
+                ts.append(a.elapsed_time(b))
+            res[name + "_ms"] = float(np.median(ts))
+        res["speedup"] = res["streaming_ms"] / res["resident_ms"]
+        res["rows"] = I
+        out[f"mode{n}"] = res
+    return out
+
+
 def config_dict(cfg):
     return {"workload": cfg.name, "dims": list(cfg.dims), "nnz_generated": cfg.nnz, "R": cfg.R,
             "seed": cfg.seed, "admm": "eps=0, max_iter=10 (PAPER.md L930-933)",
@@ -148,6 +189,9 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--ablation", action="store_true",
+                    help="also time one ADMM update per mode with the streaming (one launch per inner "
+                         "iteration, the paper's fused shape) and the row-resident variants (SURVEY f2)")
     args = ap.parse_args()
     cfg = datagen.CONFIGS[args.config]
     if args.impl == "reference":
@@ -222,9 +266,10 @@ def main():
         byts = sum(cm.mttkrp_bytes(nnz, cfg.dims, n, R) for n in range(N))
         launches_per = N   # one MTTKRP per mode per step
         ach = byts / (mtt_ms * 1e-3) / 1e9
-        roof = {"kernel": "mttkrp (k_mttkrp + carry fix-up)", "bound": "hbm", "achieved": ach,
+        roof = {"kernel": "mttkrp (k_mttkrp_fast + carry fix-up)", "bound": "hbm", "achieved": ach,
                 "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": ach / peaks["hbm_gbs"],
-                "traffic": None, "peak_source": peak_src,
+                "traffic": measured_traffic(cfg.name), "traffic_source": "profiles/r01_traffic.json (ncu, mode 0)",
+                "peak_source": peak_src,
                 "algorithmic_bytes_per_launch": byts / launches_per,
                 "avg_launch_ms": mtt_ms / launches_per,
                 "per_mode_ms": (mp[:, 1] / K).tolist()}
@@ -264,6 +309,8 @@ def main():
         line["e2e"] = {"value": float(np.mean(ts)) / 1e3, "unit": "s", "h2d_bytes_per_step": fac_bytes,
                        "d2h_bytes_per_step": fac_bytes + R * 8 + 8,
                        "note": "cstf_factorize_host: initial factors H2D, 1 outer iteration, factors+lambda+fit D2H"}
+    if args.ablation and world == 1:
+        line["ablation"] = admm_ablation(B, cfg, R, stream)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, cores, tco = oracle_outer_iteration(cfg, idx, vals, R, 1, 0)
         line["cpu_baseline"] = {"value": v, "unit": "s", "cores": cores, "kind": "oracle",

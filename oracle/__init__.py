@@ -23,6 +23,7 @@ _lib = None
 OK, EINVAL, ENOMEM, NOT_SPD, NUMERIC = 0, 1, 3, 6, 7
 PROX_NONNEG, PROX_IDENTITY, PROX_L1, PROX_NONNEG_L1 = 0, 1, 2, 3
 WARM_SCALED, WARM_NORMALIZED = 0, 1
+UPDATE_ADMM, UPDATE_HALS, UPDATE_MU = 0, 1, 2
 
 
 class OracleError(RuntimeError):
@@ -57,9 +58,11 @@ def _get():
         L.oracle_cholesky.argtypes = [i32, p, p]
         L.oracle_admm.argtypes = [i64, i32, p, p, p, p, d, i32, d, i32, d, p, p]
         L.oracle_normalize.argtypes = [i64, i32, p, p]
+        L.oracle_hals.argtypes = [i64, i32, p, p, p, i32]
+        L.oracle_mu.argtypes = [i64, i32, p, p, p, i32]
         L.oracle_fit.restype = d
         L.oracle_fit.argtypes = [i32, i32, d, i64, p, p, p, p]
-        L.oracle_factorize.argtypes = [i32, p, i64, p, p, d, i32, i32, d, d, i32, d, i32, i32, i32, d,
+        L.oracle_factorize.argtypes = [i32, p, i64, p, p, d, i32, i32, d, d, i32, d, i32, i32, i32, d, i32,
                                        p, p, p, p, p, p, p]
         _lib = L
     return _lib
@@ -214,8 +217,31 @@ def fit(normX2, M_last, H_last, lam, grams) -> float:
                                    H_last.ctypes.data, lam.ctypes.data, _ptrs(gs)))
 
 
+def hals(M, S, H, sweeps=1):
+    """f1 HALS (reading D21): column-wise non-negative coordinate updates, in order."""
+    M = _c64(M); S = _c64(S)
+    H = np.array(H, dtype=np.float64, copy=True, order="C")
+    I, R = H.shape
+    st = _get().oracle_hals(I, R, M.ctypes.data, S.ctypes.data, H.ctypes.data, int(sweeps))
+    if st:
+        raise OracleError(st, "hals")
+    return H
+
+
+def mu(M, S, H, sweeps=1):
+    """f1 MU (reading D22): h <- h * m / (h S + 1e-16)."""
+    M = _c64(M); S = _c64(S)
+    H = np.array(H, dtype=np.float64, copy=True, order="C")
+    I, R = H.shape
+    st = _get().oracle_mu(I, R, M.ctypes.data, S.ctypes.data, H.ctypes.data, int(sweeps))
+    if st:
+        raise OracleError(st, "mu")
+    return H
+
+
 def factorize(X: Tensor, factors, outer_iters=10, tol=1e-2, max_iter=10, rho=0.0,
-              warm=WARM_SCALED, normalize_init=True, prox=PROX_NONNEG, fit_tol=0.0, alpha=0.0):
+              warm=WARM_SCALED, normalize_init=True, prox=PROX_NONNEG, fit_tol=0.0, alpha=0.0,
+              update=UPDATE_ADMM):
     """O9/O11: Alg. 1 (L476-506) with readings D4, D6, D11, D13.
 
     Returns dict(factors, lam (N x R), fit[outer_done], iters[outer_done x N], phase_ms[4],
@@ -233,7 +259,7 @@ def factorize(X: Tensor, factors, outer_iters=10, tol=1e-2, max_iter=10, rho=0.0
     st = _get().oracle_factorize(N, dims_a.ctypes.data, X.nnz, _ptrs(X.idx), X.vals.ctypes.data,
                                  float(X.normX2), R, int(outer_iters), float(fit_tol), float(tol),
                                  int(max_iter), float(rho), int(warm), int(bool(normalize_init)),
-                                 int(prox), float(alpha), _ptrs(H), lam.ctypes.data, fits.ctypes.data,
+                                 int(prox), float(alpha), int(update), _ptrs(H), lam.ctypes.data, fits.ctypes.data,
                                  iters.ctypes.data, ctypes.byref(done), phase.ctypes.data,
                                  trace.ctypes.data)
     if st:

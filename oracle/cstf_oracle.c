@@ -360,6 +360,53 @@ int oracle_admm(int64_t I, int R, const double* M, const double* S, double* H, d
   return ORC_OK;
 }
 
+/* ---------------- f1: HALS and MU updates (Sec. 5.4) ---------------------
+ * The paper plugs two more non-negativity schemes into the same framework
+ * (AUNTF_GPU, L717-722) without spelling them out; readings D21 / D22:
+ *  HALS [4], one sweep per row, columns in order (Gauss-Seidel inside the row):
+ *     h_r <- max(0, h_r + (m_r - sum_k h_k S[k][r]) / S[r][r])   (S[r][r] > 0; else h_r kept)
+ *  MU [14], all columns at once from the previous h:
+ *     h_r <- h_r * m_r / (sum_k h_k S[k][r] + 1e-16)
+ * `sweeps` passes over every row. */
+#define MU_EPS 1e-16
+int oracle_hals(int64_t I, int R, const double* M, const double* S, double* H, int sweeps) {
+  if (R < 1 || R > 128 || sweeps < 1) return ORC_EINVAL;
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < I; i++) {
+    const double* m = M + i * R;
+    double* h = H + i * R;
+    for (int sw = 0; sw < sweeps; sw++)
+      for (int r = 0; r < R; r++) {
+        const double d = S[r * R + r];
+        if (!(d > 0.0)) continue;
+        double dot = 0.0;
+        for (int k = 0; k < R; k++) dot = dot + h[k] * S[k * R + r];
+        const double v = h[r] + (m[r] - dot) / d;
+        h[r] = v > 0.0 ? v : 0.0;
+      }
+  }
+  return ORC_OK;
+}
+
+int oracle_mu(int64_t I, int R, const double* M, const double* S, double* H, int sweeps) {
+  if (R < 1 || R > 128 || sweeps < 1) return ORC_EINVAL;
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < I; i++) {
+    const double* m = M + i * R;
+    double* h = H + i * R;
+    double den[128];
+    for (int sw = 0; sw < sweeps; sw++) {
+      for (int r = 0; r < R; r++) {
+        double dot = 0.0;
+        for (int k = 0; k < R; k++) dot = dot + h[k] * S[k * R + r];
+        den[r] = dot + MU_EPS;
+      }
+      for (int r = 0; r < R; r++) h[r] = h[r] * m[r] / den[r];
+    }
+  }
+  return ORC_OK;
+}
+
 /* ---------------- O8: normalize (Alg. 1 l.11, L499; readings D7, D8) ------------------
  * lambda_r = sqrt(sum_i h_ir^2); if lambda_r > 0 the column is divided by it. */
 int oracle_normalize(int64_t I, int R, double* H, double* lam) {
@@ -424,6 +471,7 @@ double oracle_fit(int N, int R, double normX2, int64_t I_last, const double* M_l
  *   H = H^(n) diag(lambda^(n)) (warm = 0, scaled, D4) or H^(n) (warm = 1, literal Alg. 1);
  *   ADMM(S, M, H, U^(n)); (H^(n), lambda^(n)) = normalize(H); G^(n) = H^(n)T H^(n)
  * then fit; stop early if fit_tol > 0 and |fit - fit_prev| < fit_tol (D11).
+ * update: 0 ADMM (Alg. 2), 1 HALS, 2 MU (f1; max_iter sweeps, S unused by rho).
  * lam_all: N*R output (every mode's lambda; the Kruskal lambda is the last mode's, D10).
  * phase_ms[4] += GRAM, MTTKRP, UPDATE, NORMALIZE wall times.
  * trace_out (optional) [outer_iters][N][max_iter][4]: the four sums of every ADMM
@@ -431,7 +479,7 @@ double oracle_fit(int N, int R, double normX2, int64_t I_last, const double* M_l
 int oracle_factorize(int N, const int64_t* dims, int64_t nnz, const int32_t* const* cidx,
                      const double* cvals, double normX2, int R, int outer_iters, double fit_tol,
                      double tol, int max_iter, double rho_in, int warm, int normalize_init, int prox,
-                     double alpha, double* const* H, double* lam_all, double* fit_out, int* iters_out,
+                     double alpha, int update, double* const* H, double* lam_all, double* fit_out, int* iters_out,
                      int* outer_done, double* phase_ms, double* trace_out) {
   if (N < 2 || N > 8 || R < 1 || R > 128 || outer_iters < 1 || max_iter < 1) return ORC_EINVAL;
   int st = ORC_OK;
@@ -469,9 +517,11 @@ int oracle_factorize(int N, const int64_t* dims, int64_t nnz, const int32_t* con
       }
       double stats[6];
       double* tr = trace_out ? trace_out + ((size_t)t * N + n) * (size_t)max_iter * 4 : NULL;
-      st = oracle_admm(dims[n], R, M, S, H[n], U[n], tol, max_iter, rho_in, prox, alpha, stats, tr);
+      if (update == 1) st = oracle_hals(dims[n], R, M, S, H[n], max_iter);
+      else if (update == 2) st = oracle_mu(dims[n], R, M, S, H[n], max_iter);
+      else st = oracle_admm(dims[n], R, M, S, H[n], U[n], tol, max_iter, rho_in, prox, alpha, stats, tr);
       if (st) break;
-      if (iters_out) iters_out[t * N + n] = (int)stats[0];
+      if (iters_out) iters_out[t * N + n] = update ? max_iter : (int)stats[0];
       double t3 = now_ms();
       oracle_normalize(dims[n], R, H[n], lam);
       double t4 = now_ms();

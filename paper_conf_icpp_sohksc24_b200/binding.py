@@ -27,6 +27,7 @@ CSTF_ERR_CUDA, CSTF_ERR_NCCL, CSTF_ERR_NOT_SPD, CSTF_ERR_NUMERIC = 4, 5, 6, 7
 CSTF_PROX_NONNEG, CSTF_PROX_IDENTITY, CSTF_PROX_L1, CSTF_PROX_NONNEG_L1 = 0, 1, 2, 3
 CSTF_ADMM_AUTO, CSTF_ADMM_STREAMING, CSTF_ADMM_RESIDENT = 0, 1, 2
 CSTF_WARM_SCALED, CSTF_WARM_NORMALIZED = 0, 1
+CSTF_UPDATE_ADMM, CSTF_UPDATE_HALS, CSTF_UPDATE_MU = 0, 1, 2
 PHASES = ("GRAM", "MTTKRP", "UPDATE", "NORMALIZE", "COMM")
 NUM_PHASES = len(PHASES)
 
@@ -53,7 +54,7 @@ class AdmmStats(ctypes.Structure):
 
 class Opts(ctypes.Structure):
     _fields_ = [("R", c_int), ("outer_iters", c_int), ("fit_tol", c_double), ("admm", AdmmOpts),
-                ("warm", c_int), ("normalize_init", c_int), ("timing", c_int)]
+                ("warm", c_int), ("normalize_init", c_int), ("timing", c_int), ("update", c_int)]
 
 
 class Report(ctypes.Structure):
@@ -93,6 +94,8 @@ _decl("cstf_gram", c_int, [c_void_p, c_int64, c_int, c_void_p, c_void_p, c_void_
 _decl("cstf_normalize", c_int, [c_void_p, c_int64, c_int, c_void_p, c_void_p, c_void_p, c_void_p])
 _decl("cstf_admm_update", c_int, [c_void_p, c_void_p, c_void_p, c_void_p, c_int64, c_int,
                                   ctypes.POINTER(AdmmOpts), c_void_p, ctypes.POINTER(AdmmStats), c_void_p])
+_decl("cstf_hals_update", c_int, [c_void_p, c_void_p, c_void_p, c_int64, c_int, c_int, c_void_p])
+_decl("cstf_mu_update", c_int, [c_void_p, c_void_p, c_void_p, c_int64, c_int, c_int, c_void_p])
 _decl("cstf_factorize", c_int, [c_void_p, ctypes.POINTER(Opts), c_void_p, c_void_p, c_void_p,
                                 ctypes.POINTER(Report), c_void_p])
 _decl("cstf_factorize_host", c_int, [c_void_p, ctypes.POINTER(Opts), c_void_p, c_void_p, c_void_p,
@@ -102,7 +105,8 @@ EXPORTED = ["cstf_status_string", "cstf_last_error_message", "cstf_version", "cs
             "cstf_comm_create", "cstf_comm_create_host", "cstf_comm_info", "cstf_comm_destroy",
             "cstf_partition_rows",
             "cstf_tensor_load_coo", "cstf_tensor_info", "cstf_tensor_export_coo", "cstf_tensor_free",
-            "cstf_mttkrp", "cstf_gram", "cstf_normalize", "cstf_admm_update", "cstf_factorize",
+            "cstf_mttkrp", "cstf_gram", "cstf_normalize", "cstf_admm_update", "cstf_hals_update",
+            "cstf_mu_update", "cstf_factorize",
             "cstf_factorize_host", "cstf_kernel_launch_count"]
 
 
@@ -323,9 +327,23 @@ def cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, rho=0.0, prox=CSTF_PROX_N
 
 def make_opts(R, outer_iters=10, fit_tol=0.0, tol=1e-2, max_iter=10, rho=0.0, prox=CSTF_PROX_NONNEG,
               variant=CSTF_ADMM_AUTO, warm=CSTF_WARM_SCALED, normalize_init=True, timing=False,
-              alpha=0.0) -> Opts:
+              alpha=0.0, update=CSTF_UPDATE_ADMM) -> Opts:
     return Opts(int(R), int(outer_iters), float(fit_tol), admm_opts(tol, max_iter, rho, prox, variant, alpha),
-                int(warm), int(bool(normalize_init)), int(bool(timing)))
+                int(warm), int(bool(normalize_init)), int(bool(timing)), int(update))
+
+
+def cstf_hals_update(M, S, H, sweeps=1, stream=None):
+    I, R = H.shape
+    _check(_lib.cstf_hals_update(_dptr(M), _dptr(S), _dptr(H), I, R, int(sweeps), _stream(stream)),
+           "cstf_hals_update")
+    return H
+
+
+def cstf_mu_update(M, S, H, sweeps=1, stream=None):
+    I, R = H.shape
+    _check(_lib.cstf_mu_update(_dptr(M), _dptr(S), _dptr(H), I, R, int(sweeps), _stream(stream)),
+           "cstf_mu_update")
+    return H
 
 
 class _ReportBufs:

@@ -73,7 +73,9 @@ __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b)
 }
 
 // RP = padded rank (multiple of 8, <= 64).  GRAM: fused Gram epilogue (RP <= 32).
-template <int RP, bool GRAM>
+// MU: multiplicative update (f1, reading D22) in the same shape: A operand = h,
+// B = S (passed in a.inv), epilogue h <- h * m / (hS + 1e-16); no dual, no sums.
+template <int RP, bool GRAM, bool MU = false>
 __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
   constexpr int NT = RP / 8;       // n-tiles of 8 columns
   constexpr int NC = 2 * NT;       // k-chunks of 4
@@ -127,7 +129,7 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
         if (rok) {
           mv = __ldcs(reinterpret_cast<const double2*>(a.M + base + col));
           hv = __ldcs(reinterpret_cast<const double2*>(a.H + base + col));
-          uv = __ldcs(reinterpret_cast<const double2*>(a.U + base + col));
+          if (!MU) uv = __ldcs(reinterpret_cast<const double2*>(a.U + base + col));
         }
         m[t][0] = mv.x; m[t][1] = mv.y; h[t][0] = hv.x; h[t][1] = hv.y; u[t][0] = uv.x; u[t][1] = uv.y;
       } else {
@@ -136,7 +138,7 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
           const bool ok = rok && (col + i) < R;
           m[t][i] = ok ? a.M[base + col + i] : 0.0;
           h[t][i] = ok ? a.H[base + col + i] : 0.0;
-          u[t][i] = ok ? a.U[base + col + i] : 0.0;
+          u[t][i] = (ok && !MU) ? a.U[base + col + i] : 0.0;
         }
       }
 #pragma unroll
@@ -152,11 +154,16 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
 #pragma unroll
       for (int c = 0; c < NC; c++) {
         const int tt = c >> 1, ii = c & 1;
-        const double av = fma(rho, h[tt][ii] + u[tt][ii], m[tt][ii]);   // M + rho (H + U)
+        const double av = MU ? h[tt][ii] : fma(rho, h[tt][ii] + u[tt][ii], m[tt][ii]);   // M + rho (H + U)
 #pragma unroll
         for (int t = 0; t < NT; t++) dmma(d[t][0], d[t][1], av, sinv[(c * NT + t) * 32 + lane]);
       }
-      if (j >= a.sums_from) {
+      if (MU) {
+#pragma unroll
+        for (int t = 0; t < NT; t++)
+#pragma unroll
+          for (int i = 0; i < 2; i++) h[t][i] = h[t][i] * m[t][i] / (d[t][i] + 1e-16);
+      } else if (j >= a.sums_from) {
         double pr = 0.0, ps = 0.0, ph = 0.0, pu = 0.0;
 #pragma unroll
         for (int t = 0; t < NT; t++)
@@ -218,11 +225,11 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
         const int col = 8 * t + 2 * q;
         if (full) {
           __stcs(reinterpret_cast<double2*>(a.Hout + base + col), make_double2(h[t][0], h[t][1]));
-          __stcs(reinterpret_cast<double2*>(a.Uout + base + col), make_double2(u[t][0], u[t][1]));
+          if (!MU) __stcs(reinterpret_cast<double2*>(a.Uout + base + col), make_double2(u[t][0], u[t][1]));
         } else {
 #pragma unroll
           for (int i = 0; i < 2; i++)
-            if (col + i < R) { a.Hout[base + col + i] = h[t][i]; a.Uout[base + col + i] = u[t][i]; }
+            if (col + i < R) { a.Hout[base + col + i] = h[t][i]; if (!MU) a.Uout[base + col + i] = u[t][i]; }
         }
       }
     }
@@ -375,6 +382,127 @@ __global__ void k_admm_decide(const double* __restrict__ sums, int j0, int k, in
   }
 }
 
+// HALS (f1, reading D21): thread per row, the row in registers, S^T in shared
+// memory (broadcast reads), columns updated in order:
+//   h_r <- max(0, h_r + (m_r mscale_r - h . S[:, r]) / S[r][r])
+// Rows are staged through a per-warp shared tile so global accesses stay coalesced.
+template <int RP>
+__global__ void __launch_bounds__(128) k_hals_rows(const double* __restrict__ M, double* __restrict__ H,
+                                                   const double* __restrict__ S, const double* __restrict__ mscale,
+                                                   const double* __restrict__ hscale, int64_t I, int R, int sweeps,
+                                                   const int* __restrict__ flag) {
+  constexpr int LD = RP + 1;                 // padded row stride in the tiles
+  extern __shared__ double sm[];
+  double* ST = sm;                           // [RP][RP]: ST[r][k] = S[k][r]
+  double* tiles = sm + RP * RP;              // [warp][2][32][LD]: h, m
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  double* th = tiles + (size_t)warp * 2 * 32 * LD;
+  double* tm = th + 32 * LD;
+  for (int x = threadIdx.x; x < RP * RP; x += blockDim.x) {
+    const int r = x / RP, k = x % RP;
+    ST[x] = (r < R && k < R) ? S[k * R + r] : 0.0;
+  }
+  __syncthreads();
+  if (*flag) return;
+  const int64_t ntiles = (I + 31) / 32;
+  for (int64_t tl = (int64_t)blockIdx.x * 4 + warp; tl < ntiles; tl += (int64_t)gridDim.x * 4) {
+    const int64_t r0 = tl * 32;
+    for (int x = lane; x < 32 * RP; x += 32) {           // coalesced tile loads
+      const int rr = x / RP, c = x % RP;
+      const bool ok = r0 + rr < I && c < R;
+      th[rr * LD + c] = ok ? H[(r0 + rr) * R + c] * (hscale ? hscale[c] : 1.0) : 0.0;
+      tm[rr * LD + c] = ok ? M[(r0 + rr) * R + c] * (mscale ? mscale[c] : 1.0) : 0.0;
+    }
+    __syncwarp();
+    double h[RP];
+#pragma unroll
+    for (int k = 0; k < RP; k++) h[k] = th[lane * LD + k];
+    for (int sw = 0; sw < sweeps; sw++) {
+#pragma unroll
+      for (int r = 0; r < RP; r++) {
+        const double d = ST[r * RP + r];
+        double dot = 0.0;
+#pragma unroll
+        for (int k = 0; k < RP; k++) dot = fma(h[k], ST[r * RP + k], dot);
+        if (d > 0.0) {
+          const double v = h[r] + (tm[lane * LD + r] - dot) / d;
+          h[r] = v > 0.0 ? v : 0.0;
+        }
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < RP; k++) th[lane * LD + k] = h[k];
+    __syncwarp();
+    for (int x = lane; x < 32 * RP; x += 32) {
+      const int rr = x / RP, c = x % RP;
+      if (r0 + rr < I && c < R) H[(r0 + rr) * R + c] = th[rr * LD + c];
+    }
+    __syncwarp();
+  }
+}
+
+// R in (64, 128]: the same update with the row kept in the shared tile (runtime loops).
+__global__ void __launch_bounds__(64) k_hals_rows_smem(const double* __restrict__ M, double* __restrict__ H,
+                                                        const double* __restrict__ S, const double* __restrict__ mscale,
+                                                        const double* __restrict__ hscale, int64_t I, int R, int sweeps,
+                                                        const int* __restrict__ flag) {
+  const int LD = R + 1;
+  extern __shared__ double sm[];
+  double* ST = sm;                           // [R][R]: ST[r][k] = S[k][r]
+  double* tiles = sm + R * R;                // [warp][2][32][LD]
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  double* th = tiles + (size_t)warp * 2 * 32 * LD;
+  double* tm = th + 32 * LD;
+  for (int x = threadIdx.x; x < R * R; x += blockDim.x) ST[x] = S[(x % R) * R + x / R];
+  __syncthreads();
+  if (*flag) return;
+  const int nw = blockDim.x >> 5;
+  const int64_t ntiles = (I + 31) / 32;
+  for (int64_t tl = (int64_t)blockIdx.x * nw + warp; tl < ntiles; tl += (int64_t)gridDim.x * nw) {
+    const int64_t r0 = tl * 32;
+    for (int x = lane; x < 32 * R; x += 32) {
+      const int rr = x / R, c = x % R;
+      const bool ok = r0 + rr < I;
+      th[rr * LD + c] = ok ? H[(r0 + rr) * R + c] * (hscale ? hscale[c] : 1.0) : 0.0;
+      tm[rr * LD + c] = ok ? M[(r0 + rr) * R + c] * (mscale ? mscale[c] : 1.0) : 0.0;
+    }
+    __syncwarp();
+    double* h = th + lane * LD;
+    for (int sw = 0; sw < sweeps; sw++)
+      for (int r = 0; r < R; r++) {
+        const double d = ST[r * R + r];
+        double dot = 0.0;
+        for (int k = 0; k < R; k++) dot = fma(h[k], ST[r * R + k], dot);
+        if (d > 0.0) {
+          const double v = h[r] + (tm[lane * LD + r] - dot) / d;
+          h[r] = v > 0.0 ? v : 0.0;
+        }
+      }
+    __syncwarp();
+    for (int x = lane; x < 32 * R; x += 32) {
+      const int rr = x / R, c = x % R;
+      if (r0 + rr < I) H[(r0 + rr) * R + c] = th[rr * LD + c];
+    }
+    __syncwarp();
+  }
+}
+
+template <int RP>
+cstf_status launch_hals_t(const double* M, double* H, const double* S, const double* mscale, const double* hscale,
+                          int64_t I, int R, int sweeps, const int* flag, cudaStream_t st) {
+  const size_t smem = (size_t)RP * RP * 8 + (size_t)4 * 2 * 32 * (RP + 1) * 8;
+  static bool attr = false;
+  if (!attr) {
+    CSTF_CUDA(cudaFuncSetAttribute(k_hals_rows<RP>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = true;
+  }
+  const int64_t ntiles = (I + 31) / 32;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((ntiles + 3) / 4, (int64_t)device_info().sms * 4));
+  k_hals_rows<RP><<<grid, 128, smem, st>>>(M, H, S, mscale, hscale, I, R, sweeps, flag);
+  CSTF_LAUNCHED();
+  return CSTF_OK;
+}
+
 struct Workspace {
   DevBuf slots, sums, out, hs[2], us[2], gpart;
   double* host_out = nullptr;
@@ -394,19 +522,19 @@ size_t dmma_smem(int RP, bool gram, int nsl) {
          (gram ? (size_t)kWarpsA * NT * (NT + 1) / 2 * 64 * 8 : 0);
 }
 
-template <int RP, bool GRAM>
+template <int RP, bool GRAM, bool MU = false>
 cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
   const int nsl = k.kiters - k.sums_from;
   const size_t smem = dmma_smem(RP, GRAM, nsl);
   static int per_sm[kMaxK + 1] = {0};
   static bool attr = false;
   if (!attr) {
-    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM, MU>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)dmma_smem(RP, GRAM, kMaxK)));
     attr = true;
   }
   if (!per_sm[nsl]) {
-    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM>, kThreads, smem));
+    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM, MU>, kThreads, smem));
     if (per_sm[nsl] < 1) per_sm[nsl] = 1;
   }
   const int64_t groups = (k.I + 7) / 8;
@@ -414,7 +542,7 @@ cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
   const int64_t cap = (int64_t)device_info().sms * per_sm[nsl];
   if (g > cap) g = cap;
   grid = (int)(g < 1 ? 1 : g);
-  k_admm_dmma<RP, GRAM><<<grid, kThreads, smem, st>>>(k);
+  k_admm_dmma<RP, GRAM, MU><<<grid, kThreads, smem, st>>>(k);
   CSTF_LAUNCHED();
   return CSTF_OK;
 }
@@ -458,6 +586,72 @@ cstf_status launch_kernel(const KArgs& k, int& grid, bool gram, cudaStream_t st)
 }  // namespace
 
 bool admm_can_fuse_gram(int R, double tol) { return tol == 0.0 && R <= 32; }
+
+cstf_status hals_run(const UpdArgs& A, cudaStream_t st) {
+  switch ((A.R + 7) & ~7) {
+#define C(RP) case RP: return launch_hals_t<RP>(A.M, A.H, A.S, A.mscale, A.hscale, A.I, A.R, A.sweeps, A.flag, st);
+    C(8) C(16) C(24) C(32)
+#undef C
+    default: break;   // R > 32: row kept in the shared tile
+  }
+  const int nw = A.R > 64 ? 1 : 2;     // warps per CTA so S^T + tiles fit shared memory
+  const size_t smem = (size_t)A.R * A.R * 8 + (size_t)nw * 2 * 32 * (A.R + 1) * 8;
+  static bool attr = false;
+  if (!attr) {
+    CSTF_CUDA(cudaFuncSetAttribute(k_hals_rows_smem, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                   (int)((size_t)128 * 128 * 8 + (size_t)2 * 32 * 129 * 8)));
+    attr = true;
+  }
+  const int64_t ntiles = (A.I + 31) / 32;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((ntiles + nw - 1) / nw, (int64_t)device_info().sms * 4));
+  k_hals_rows_smem<<<grid, 32 * nw, smem, st>>>(A.M, A.H, A.S, A.mscale, A.hscale, A.I, A.R, A.sweeps, A.flag);
+  CSTF_LAUNCHED();
+  return CSTF_OK;
+}
+
+// MU on the DMMA path (R <= 64); the Gram of the result is fused when R <= 32.
+cstf_status mu_run(const UpdArgs& A, cudaStream_t st) {
+  const int RP = (A.R + 7) & ~7;
+  if (RP > 64) return fail(CSTF_ERR_UNSUPPORTED, "MU update for R > 64");
+  Workspace& w = ws();
+  const int maxgrid = device_info().sms * 8;
+  CSTF_TRY(w.slots.ensure((size_t)kMaxK * maxgrid * 4 * 8));
+  const bool gram = A.G != nullptr && A.R <= 32;
+  if (gram) CSTF_TRY(w.gpart.ensure((size_t)maxgrid * 10 * 64 * 8));
+  KArgs k{};
+  k.M = A.M; k.H = A.H; k.U = nullptr; k.Hout = A.H; k.Uout = nullptr;
+  k.hscale = A.hscale; k.mscale = A.mscale; k.I = A.I; k.R = A.R; k.inv = A.S; k.scal = A.scal;
+  k.flag = A.flag; k.prox = 0; k.alpha = 0.0; k.slots = w.slots.as<double>();
+  k.gpart = gram ? w.gpart.as<double>() : nullptr;
+  for (int j0 = 0; j0 < A.sweeps; j0 += kMaxK) {
+    const int kk = std::min(kMaxK, A.sweeps - j0);
+    const bool last = j0 + kk >= A.sweeps;
+    k.kiters = kk;
+    k.sums_from = kk;
+    if (j0 > 0) k.hscale = nullptr;
+    const bool g = gram && last;
+    k.gpart = g ? w.gpart.as<double>() : nullptr;
+    int grid = 0;
+    cstf_status s = CSTF_OK;
+    switch (RP) {
+      case 8: s = g ? launch_dmma_t<8, true, true>(k, grid, st) : launch_dmma_t<8, false, true>(k, grid, st); break;
+      case 16: s = g ? launch_dmma_t<16, true, true>(k, grid, st) : launch_dmma_t<16, false, true>(k, grid, st); break;
+      case 24: s = g ? launch_dmma_t<24, true, true>(k, grid, st) : launch_dmma_t<24, false, true>(k, grid, st); break;
+      case 32: s = g ? launch_dmma_t<32, true, true>(k, grid, st) : launch_dmma_t<32, false, true>(k, grid, st); break;
+      case 40: s = launch_dmma_t<40, false, true>(k, grid, st); break;
+      case 48: s = launch_dmma_t<48, false, true>(k, grid, st); break;
+      case 56: s = launch_dmma_t<56, false, true>(k, grid, st); break;
+      case 64: s = launch_dmma_t<64, false, true>(k, grid, st); break;
+    }
+    CSTF_TRY(s);
+    if (g) {
+      const int NT = RP / 8;
+      k_gram_from_parts<<<NT * (NT + 1) / 2 * 64, 256, 0, st>>>(w.gpart.as<double>(), grid, NT, A.R, A.G);
+      CSTF_LAUNCHED();
+    }
+  }
+  return CSTF_OK;
+}
 
 // Runs one ADMM update.  tol == 0: chunks of up to kMaxK iterations in place,
 // no host round trip until the end; the final chunk can also emit the Gram of

@@ -35,7 +35,7 @@ bool rank_ok(int R) { return R >= 1 && R <= 128; }
 
 // Device-side scratch of one factorize / admm_update call, cached per device.
 struct DriverWs {
-  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8];
+  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8], S;
   double* host_small = nullptr;  // pinned: fit, flags
   cudaStream_t side = nullptr;   // the R x R step of a mode overlaps its MTTKRP
   cudaEvent_t fork = nullptr, join = nullptr;
@@ -112,6 +112,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
   if (o->admm.prox < CSTF_PROX_NONNEG || o->admm.prox > CSTF_PROX_NONNEG_L1 || !(o->admm.alpha >= 0.0))
     return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
+  if (o->update < CSTF_UPDATE_ADMM || o->update > CSTF_UPDATE_MU) return fail(CSTF_ERR_INVALID_ARG, "unknown update");
+  if (o->update == CSTF_UPDATE_MU && R > 64) return fail(CSTF_ERR_UNSUPPORTED, "MU update for R > 64");
   const bool dist = X->nranks > 1;
   if (comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
     return fail(CSTF_ERR_INVALID_ARG, "comm does not match the tensor's partition");
@@ -144,6 +146,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
   CSTF_TRY(w.lam.ensure((size_t)N * R * 8));
   CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
+  CSTF_TRY(w.S.ensure((size_t)R * R * 8));
   CSTF_TRY(w.scal.ensure((size_t)(8 + 2 * R) * 8));
   CSTF_TRY(w.flag.ensure(64));
   CSTF_TRY(w.fitbuf.ensure(300 * 8));
@@ -198,7 +201,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       CSTF_CUDA(cudaEventRecord(w.fork, st));
       CSTF_CUDA(cudaStreamWaitEvent(w.side, w.fork, 0));
       CSTF_TRY(chol_inverse(nullptr, G, N, n, R, o->admm.rho, w.inv.as<double>(), w.scal.as<double>(), flag,
-                            w.side, lam, colscale));
+                            w.side, lam, colscale, w.S.as<double>()));
       CSTF_CUDA(cudaEventRecord(w.join, w.side));
       // a2: MTTKRP of the raw factors (MTTKRP phase = both, overlapped)
       tm.begin(n, CSTF_PHASE_MTTKRP);
@@ -214,10 +217,25 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       a.I = I; a.R = R; a.inv = w.inv.as<double>(); a.scal = w.scal.as<double>(); a.flag = flag;
       a.tol = o->admm.tol; a.max_iter = o->admm.max_iter; a.prox = o->admm.prox; a.variant = o->admm.variant;
       a.alpha = o->admm.alpha;
-      const bool fused = admm_can_fuse_gram(R, o->admm.tol);
-      a.G = fused ? Gn : nullptr;      // a7 fused into the ADMM epilogue
+      bool fused = false;
       int iters = 0;
-      CSTF_TRY(admm_run(a, comm, st, nullptr, &iters, nullptr));
+      if (o->update == CSTF_UPDATE_ADMM) {
+        fused = admm_can_fuse_gram(R, o->admm.tol);
+        a.G = fused ? Gn : nullptr;      // a7 fused into the ADMM epilogue
+        CSTF_TRY(admm_run(a, comm, st, nullptr, &iters, nullptr));
+      } else {                           // f1: HALS / MU on the same M, S
+        UpdArgs u;
+        u.M = M; u.H = Hn; u.S = w.S.as<double>(); u.mscale = colscale; u.hscale = a.hscale;
+        u.flag = flag; u.I = I; u.R = R; u.sweeps = o->admm.max_iter;
+        if (o->update == CSTF_UPDATE_MU) {
+          fused = R <= 32;
+          u.G = fused ? Gn : nullptr;
+          CSTF_TRY(mu_run(u, st));
+        } else {
+          CSTF_TRY(hals_run(u, st));
+        }
+        iters = o->admm.max_iter;
+      }
       if (rep && rep->admm_iters) rep->admm_iters[t * N + n] = iters;
       tm.end(n, CSTF_PHASE_UPDATE);
       // a7 (when not fused): raw Gram; a6: lambda and the normalised Gram
@@ -368,6 +386,29 @@ cstf_status cstf_admm_update(const double* d_M, const double* d_S, double* d_H, 
   CSTF_TRY(check_flag(flag, st));
   if (host_stats) *host_stats = stats;
   return CSTF_OK;
+}
+
+static cstf_status run_update(int kind, const double* d_M, const double* d_S, double* d_H, int64_t I, int R,
+                              int sweeps, void* stream) {
+  if (!d_S || I < 0 || (I > 0 && (!d_M || !d_H))) return fail(CSTF_ERR_INVALID_ARG, "NULL argument or I < 0");
+  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+  if (sweeps < 1) return fail(CSTF_ERR_INVALID_ARG, "sweeps < 1");
+  DriverWs& w = dws();
+  CSTF_TRY(w.flag.ensure(64));
+  CSTF_CUDA(cudaMemsetAsync(w.flag.p, 0, 4, S(stream)));
+  UpdArgs u;
+  u.M = d_M; u.H = d_H; u.S = d_S; u.flag = w.flag.as<int>(); u.I = I; u.R = R; u.sweeps = sweeps;
+  return kind == CSTF_UPDATE_MU ? mu_run(u, S(stream)) : hals_run(u, S(stream));
+}
+
+cstf_status cstf_hals_update(const double* d_M, const double* d_S, double* d_H, int64_t I, int R, int sweeps,
+                             void* stream) {
+  return run_update(CSTF_UPDATE_HALS, d_M, d_S, d_H, I, R, sweeps, stream);
+}
+
+cstf_status cstf_mu_update(const double* d_M, const double* d_S, double* d_H, int64_t I, int R, int sweeps,
+                           void* stream) {
+  return run_update(CSTF_UPDATE_MU, d_M, d_S, d_H, I, R, sweeps, stream);
 }
 
 cstf_status cstf_factorize(const cstf_tensor* X, const cstf_opts* opts, const cstf_comm* comm,

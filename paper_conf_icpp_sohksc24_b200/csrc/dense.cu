@@ -171,7 +171,8 @@ __global__ void k_fill(double* __restrict__ d, int64_t n, double v) {
 __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __restrict__ grams,
                                int N, int skip, int R, double rho_in, double* __restrict__ Linv,
                                double* __restrict__ Inv, double* __restrict__ scal, int* flag,
-                               const double* __restrict__ lam, double* __restrict__ colscale) {
+                               const double* __restrict__ lam, double* __restrict__ colscale,
+                               double* __restrict__ S_out) {
   if (lam) {
     for (int r = threadIdx.x; r < R; r += blockDim.x) {
       double ms = 1.0;
@@ -205,6 +206,7 @@ __global__ void k_chol_inverse(const double* __restrict__ S_in, const double* __
       v = S_in[e];
     }
     L[e] = v;
+    if (S_out) S_out[e] = v;
   }
   __syncthreads();
   if (threadIdx.x == 0) {
@@ -400,7 +402,7 @@ cstf_status gram_to_lambda(double* d_G, int R, double* d_lam, cudaStream_t st) {
 
 cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int skip, int R,
                          double rho_in, double* d_inv, double* d_scal, int* d_flag,
-                         cudaStream_t st, const double* d_lam, double* d_colscale) {
+                         cudaStream_t st, const double* d_lam, double* d_colscale, double* d_S_out) {
   Workspace& w = ws();
   CSTF_TRY(w.linv.ensure((size_t)R * R * 8));
   const size_t smem = (size_t)R * R * 8 * (R <= 64 ? 2 : 1);
@@ -410,7 +412,7 @@ cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int sk
     attr_set = true;
   }
   k_chol_inverse<<<1, 256, smem, st>>>(d_S, d_grams, N, skip, R, rho_in, w.linv.as<double>(), d_inv,
-                                       d_scal, d_flag, d_lam, d_colscale);
+                                       d_scal, d_flag, d_lam, d_colscale, d_S_out);
   CSTF_LAUNCHED();
   return CSTF_OK;
 }

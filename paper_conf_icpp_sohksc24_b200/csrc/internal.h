@@ -169,7 +169,8 @@ cstf_status fill(double* d, int64_t n, double v, cudaStream_t st);
 // prod_{k != skip} 1/lambda_k (0 where lambda_k = 0) and d_colscale[R..2R) = 1/lambda_skip.
 cstf_status chol_inverse(const double* d_S, const double* d_grams, int N, int skip, int R,
                          double rho_in, double* d_inv, double* d_scal, int* d_flag,
-                         cudaStream_t st, const double* d_lam = nullptr, double* d_colscale = nullptr);
+                         cudaStream_t st, const double* d_lam = nullptr, double* d_colscale = nullptr,
+                         double* d_S_out = nullptr);
 // lambda_r = sqrt(G_rr); G <- D^-1 G D^-1 (H untouched)
 cstf_status gram_to_lambda(double* d_G, int R, double* d_lam, cudaStream_t st);
 // fit (D12): writes d_out[0] = fit.  inner = sum_i sum_r M_ir H_ir colw_r, xhat = lam^T (*G) lam.
@@ -203,5 +204,22 @@ struct AdmmArgs {
 cstf_status admm_run(const AdmmArgs& a, const cstf_comm* comm, cudaStream_t st,
                      cstf_admm_stats* stats, int* iters_out, int64_t* launches);
 bool admm_can_fuse_gram(int R, double tol);
+
+// f1 update schemes (HALS / MU), same row-wise shape as ADMM
+struct UpdArgs {
+  const double* M;
+  double* H;
+  const double* S;        // R x R Hadamard of Grams
+  const double* mscale = nullptr;
+  const double* hscale = nullptr;
+  const double* scal = nullptr;   // unused by HALS/MU (rho slot)
+  const int* flag;
+  double* G = nullptr;    // MU: fused raw Gram of the result (R <= 32)
+  int64_t I;
+  int R;
+  int sweeps;
+};
+cstf_status hals_run(const UpdArgs& a, cudaStream_t st);
+cstf_status mu_run(const UpdArgs& a, cudaStream_t st);
 
 }  // namespace cstf

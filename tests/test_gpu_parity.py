@@ -370,3 +370,34 @@ def test_factorize_nonneg_l1(B):
     n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
     assert tie is None
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+
+
+@pytest.mark.parametrize("update", ["hals", "mu"])
+@pytest.mark.parametrize("I,R", [(1, 8), (1003, 8), (3001, 32), (999, 64), (300, 100)])
+def test_hals_mu_updates(B, update, I, R):
+    """f1: one HALS / MU update (3 sweeps) vs the oracle on positive data."""
+    if update == "mu" and R > 64:
+        pytest.skip("MU is built for R <= 64")
+    M, S, H, U = admm_inputs(I, R, 5 + R)
+    M = np.abs(M)
+    Hd = cu(H)
+    getattr(B, f"cstf_{update}_update")(cu(M), cu(S), Hd, sweeps=3)
+    ref = getattr(oracle, update)(M, S, H, sweeps=3)
+    assert normwise(host(Hd), ref) <= TOL
+    assert np.min(host(Hd)) >= 0.0
+
+
+@pytest.mark.parametrize("update,R", [(1, 16), (2, 16), (1, 40), (2, 40)])
+def test_factorize_hals_mu(B, update, R):
+    c = datagen.CONFIGS["enron"].scaled(60, nnz_factor=2000)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, R, c.seed)
+    ref = oracle.coalesce(c.dims, idx, vals)
+    orc = oracle.factorize(ref, start, outer_iters=5, max_iter=2, update=update)
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    F = [cu(f) for f in start]
+    lam = cu(np.zeros(R))
+    gpu = B.cstf_factorize(X, F, lam, B.make_opts(R, outer_iters=5, max_iter=2, update=update))
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+    for a, b in zip(F, orc["factors"]):
+        assert normwise(host(a), b) <= 1e-6

@@ -444,3 +444,61 @@ def test_f3_l1_with_zero_alpha_is_the_plain_operator(rng):
     a = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), max_iter=20, prox=oracle.PROX_NONNEG_L1, alpha=0.0)
     b = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), max_iter=20, prox=oracle.PROX_NONNEG)
     assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+
+
+# --------------------------------------------------------------------- f1: HALS / MU
+def nnls_objective(S, M, H):
+    return float(np.sum(0.5 * np.einsum("ir,rs,is->i", H, S, H) - np.einsum("ir,ir->i", M, H)))
+
+
+@pytest.mark.parametrize("R", [2, 3, 4])
+def test_f1_hals_converges_to_nnls(rng, R):
+    """HALS is exact coordinate descent on the per-row NNLS: it reaches the brute-force minimiser."""
+    S = make_S(rng, R)
+    I = 40
+    M = (rng.random((I, R)) - 0.45) * np.diag(S).mean()
+    H = oracle.hals(M, S, np.zeros((I, R)) + 0.1, sweeps=3000)
+    ref = np.array([nnls_bruteforce(S, M[i]) for i in range(I)])
+    assert normwise(H, ref) <= 1e-9
+
+
+@pytest.mark.parametrize("update", ["hals", "mu"])
+def test_f1_monotone_objective(rng, update):
+    """Both schemes never increase the NNLS objective (Lee-Seung for MU; exact
+    coordinate minimisation for HALS) on non-negative data."""
+    R, I = 6, 200
+    S = make_S(rng, R)
+    M = rng.random((I, R)) * np.diag(S).mean()
+    H = rng.random((I, R))
+    f = getattr(oracle, update)
+    prev = nnls_objective(S, M, H)
+    for _ in range(30):
+        H = f(M, S, H, sweeps=1)
+        cur = nnls_objective(S, M, H)
+        assert cur <= prev + 1e-12 * abs(prev)
+        prev = cur
+    assert np.min(H) >= 0.0
+
+
+def test_f1_mu_fixed_point_kkt(rng):
+    """MU's fixed points satisfy h_r (HS - M)_r = 0; from a positive start on positive
+    data it approaches the NNLS solution."""
+    R, I = 3, 30
+    S = make_S(rng, R)
+    M = rng.random((I, R)) * np.diag(S).mean()
+    H = oracle.mu(M, S, np.ones((I, R)), sweeps=20000)
+    G = H @ S - M
+    assert np.max(np.abs(H * G)) <= 1e-6 * np.max(np.abs(M))
+    ref = np.array([nnls_bruteforce(S, M[i]) for i in range(I)])
+    assert normwise(H, ref) <= 1e-3
+
+
+def test_f1_factorize_schemes_on_planted(rng):
+    """The planted rank-8 tensor is fitted by all three schemes (HALS/MU slower than ADMM)."""
+    p = datagen.planted_tiny(1)
+    X = oracle.coalesce(p.dims, p.idx, p.vals)
+    start = datagen.perturbed_start(p, 1)
+    for upd in (oracle.UPDATE_HALS, oracle.UPDATE_MU):
+        r = oracle.factorize(X, start, outer_iters=30, max_iter=1, update=upd)
+        assert r["fit"][-1] > 0.99
+        assert np.all(np.diff(r["fit"]) > -1e-9)

@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libcstf.so")
+LIB_PATH = os.environ.get("CSTF_LIB") or os.path.join(_HERE, "lib", "libcstf.so")   # override: experiments
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"libcstf.so not built ({LIB_PATH}); run "
                       "`python -m paper_conf_icpp_sohksc24_b200.build` (no CPU fallback exists)")

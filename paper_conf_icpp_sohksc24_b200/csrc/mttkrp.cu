@@ -190,8 +190,9 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
   }
 }
 
-template <int NOTHER, int R, int RECB>
-__global__ void __launch_bounds__(kWarps * 32, 2) k_mttkrp_fast(MArgs a) {
+// MINB: CTAs per SM the register budget targets (2 for long rows, 4 for short ones)
+template <int NOTHER, int R, int RECB, int MINB>
+__global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
   constexpr int G = (R / 2) < 32 ? (R / 2) : 32;
   const int gl = (threadIdx.x & 31) % G;
   const char* Fb[NOTHER];
@@ -343,6 +344,9 @@ bool launch_tiled_r(const MArgs& a, int grid, cudaStream_t st) {
 
 template <int NOTHER, int RECB>
 bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled) {
+  // short rows (few nonzeros per row): row flushes dominate and latency hiding
+  // needs more warps -> the 4-CTA/SM register budget; long rows -> 2 CTAs/SM
+  const bool short_rows = a.nnz < 64 * a.I;
   if (tiled) {
     switch (a.R) {     // slab = 256 rows x R doubles: 2 KB .. 128 KB
       case 8: return launch_tiled_r<NOTHER, RECB, 8>(a, grid, st);
@@ -353,7 +357,11 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled) {
     }
   }
   switch (a.R) {
-#define CASE(RR) case RR: k_mttkrp_fast<NOTHER, RR, RECB><<<grid, kWarps * 32, 0, st>>>(a); return true;
+#define CASE(RR)                                                                     \
+  case RR:                                                                           \
+    if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4><<<grid, kWarps * 32, 0, st>>>(a); \
+    else k_mttkrp_fast<NOTHER, RR, RECB, 2><<<grid, kWarps * 32, 0, st>>>(a);           \
+    return true;
     CASE(2) CASE(4) CASE(8) CASE(16) CASE(32) CASE(64) CASE(128)
 #undef CASE
     default: return false;

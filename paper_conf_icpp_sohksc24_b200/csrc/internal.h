@@ -98,7 +98,8 @@ int comm_rank(const cstf_comm* c);
 // rowptr has nblk * I + 1 entries; MTTKRP writes one partial row per virtual row
 // and sums the partials over kb in fixed order.  The factor rows of block kb are
 // staged in shared memory by the CTA that processes them.
-constexpr int kTileRows = 256;
+constexpr int kTileRows = 256;        // SMEM-slab blocks (opt-in CSTF_KBLOCK=1)
+constexpr int64_t kL2Rows = 131072;     // L2 blocks: 32 MB of factor rows at R = 32
 struct ModeStore {
   int64_t I = 0;            // rows of this mode (local rows when distributed)
   int64_t nnz = 0;          // nonzeros in this copy
@@ -108,6 +109,9 @@ struct ModeStore {
   int other[7];             // mode id of record slot q (slot 0 = shortest other mode)
   // k-blocking
   bool tiled = false;
+  bool slab = false;        // blocks of kTileRows staged in SMEM (else L2-sized blocks)
+  int64_t blk_rows = 0;     // rows of the blocked mode per block
+  int tslot = 0;            // record slot of the blocked mode
   int64_t nblk = 1;         // blocks of the tiled mode
   int64_t Ivirt = 0;        // rows of rowptr (= I when not tiled)
   // cached work split of a tiled copy: warp-chunk starts and the block of each CTA chunk

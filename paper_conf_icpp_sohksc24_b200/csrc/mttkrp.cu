@@ -458,7 +458,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.wstart = nullptr;
   a.ckb = nullptr;
   int64_t chunk = 0, nchunks = 0;
-  if (ms.tiled) {
+  if (ms.tiled && ms.slab) {
     CSTF_TRY(tiled_split(ms, st));
     nchunks = ms.nwchunks;
     a.wstart = ms.wstart.as<int64_t>();
@@ -466,7 +466,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   } else {
     // chunk: ~4 chunks per resident warp, multiple of 32, in [256, 8192]
     const int64_t resident = (int64_t)di.sms * 8 * kWarps;
-    chunk = (nnz + resident * 4 - 1) / (resident * 4);
+    chunk = (nnz + resident * 4 - 1) / (resident * 4);   // (virtual rows when L2-blocked)
     chunk = ((chunk + 31) / 32) * 32;
     if (chunk < 256) chunk = 256;
     if (chunk > 8192) chunk = 8192;
@@ -485,7 +485,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.recb = ms.recb;
   a.nother = N - 1;
   for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
-  a.It = X->dims[ms.other[N - 2]];
+  a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor
   a.I = ms.Ivirt;
   a.nnz = nnz;
   a.chunk = chunk;
@@ -506,6 +506,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   }
   const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
   const int tgrid = (int)std::min<int64_t>(std::max<int64_t>(ms.nctachunks, 1), (int64_t)di.sms * 2);
+  // (a.ckb is set only for SMEM-slab copies; L2-blocked copies run the flat kernel on virtual rows)
   CSTF_TRY(launch_main(a, grid, tgrid, st));
   nl++;
   if (nchunks > 1) {

@@ -233,10 +233,10 @@ cstf_status lsd_sort(const int32_t* const* keys, const int64_t* dims, int nk, in
 }
 
 __global__ void k_block_keys(const int32_t* __restrict__ idx_t, const int32_t* __restrict__ idx_n, int64_t n,
-                             int64_t I, int32_t* __restrict__ kb, int32_t* __restrict__ vrow) {
+                             int64_t I, int64_t blk, int32_t* __restrict__ kb, int32_t* __restrict__ vrow) {
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
        p += (int64_t)gridDim.x * blockDim.x) {
-    const int32_t b = idx_t[p] / kTileRows;
+    const int32_t b = (int32_t)(idx_t[p] / blk);
     kb[p] = b;
     vrow[p] = (int32_t)((int64_t)b * I + idx_n[p]);
   }
@@ -561,13 +561,38 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     for (int m = 0; m < N; m++)
       if (m != n_) ms.other[k++] = m;
     std::stable_sort(ms.other, ms.other + (N - 1), [&](int a, int b) { return X->dims[a] < X->dims[b]; });
-    // k-blocking decision (host logic): short output mode, long other mode,
-    // enough nonzeros per partial row, bounded partial-row count
-    const int t = ms.other[N - 2];
-    const int64_t nblk = (X->dims[t] + kTileRows - 1) / kTileRows;
+    // Blocking decision (host logic).
+    //  * L2 blocks (opt-in CSTF_L2_BLOCK_ROWS): block the largest other factor that does not fit
+    //    in L2 (> 2 kL2Rows rows) into kL2Rows-row blocks, if the partial rows
+    //    (nblk * I_n) stay within budget and average >= 4 nonzeros each, so the
+    //    gathered slice of that factor stays L2-resident while its nonzeros stream.
+    //  * SMEM slabs (opt-in CSTF_KBLOCK=1): kTileRows-row blocks of the longest
+    //    other mode, staged in shared memory by the CTA.
     static const bool kblock_on = getenv("CSTF_KBLOCK") && atoi(getenv("CSTF_KBLOCK")) > 0;
-    ms.tiled = kblock_on && N >= 3 && nblk >= 2 && nblk * ms.I <= ((int64_t)4 << 20) && nout >= 8 * nblk * ms.I;
-    ms.nblk = ms.tiled ? nblk : 1;
+    ms.tiled = false;
+    ms.slab = false;
+    ms.nblk = 1;
+    int t = -1;
+    if (N >= 3 && kblock_on) {
+      t = ms.other[N - 2];
+      const int64_t nb = (X->dims[t] + kTileRows - 1) / kTileRows;
+      if (nb >= 2 && nb * ms.I <= ((int64_t)4 << 20) && nout >= 8 * nb * ms.I) {
+        ms.tiled = ms.slab = true; ms.blk_rows = kTileRows; ms.nblk = nb; ms.tslot = N - 2;
+      }
+    } else if (N >= 3 && getenv("CSTF_L2_BLOCK_ROWS")) {
+      // opt-in: measured slower on Delicious (the other HBM-sized factor still
+      // streams from DRAM; partial rows add traffic), DESIGN.md "MTTKRP"
+      const char* ov = getenv("CSTF_L2_BLOCK_ROWS");
+      const int64_t l2rows = atoll(ov) > 0 ? atoll(ov) : kL2Rows;
+      for (int q = N - 2; q >= 0 && !ms.tiled; q--) {     // largest other factor first
+        const int tm = ms.other[q];
+        const int64_t nb = (X->dims[tm] + l2rows - 1) / l2rows;
+        if (X->dims[tm] > 2 * l2rows && nb * ms.I <= ((int64_t)16 << 20) && nout >= 4 * nb * ms.I) {
+          ms.tiled = true; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = q; t = tm;
+        }
+      }
+    }
+    const int64_t nblk = ms.nblk;
     ms.Ivirt = ms.nblk * ms.I;
     const int32_t* keys[9];
     int64_t kd[9];
@@ -577,7 +602,7 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
       CSTF_TRY(kbk.alloc((size_t)nout * 4));
       CSTF_TRY(vrow.alloc((size_t)nout * 4));
       k_block_keys<<<grid_for(nout), kThreads, 0, st>>>(c_idx[t].as<int32_t>(), c_idx[n_].as<int32_t>(), nout,
-                                                        ms.I, kbk.as<int32_t>(), vrow.as<int32_t>());
+                                                        ms.I, ms.blk_rows, kbk.as<int32_t>(), vrow.as<int32_t>());
       CSTF_LAUNCHED();
       keys[nk] = kbk.as<int32_t>(); kd[nk++] = nblk;
     }

@@ -401,3 +401,27 @@ def test_factorize_hals_mu(B, update, R):
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
     for a, b in zip(F, orc["factors"]):
         assert normwise(host(a), b) <= 1e-6
+
+
+@pytest.mark.parametrize("R", [16, 32, 5])
+def test_mttkrp_l2_blocked_copies(B, R, monkeypatch):
+    """L2-blocked copies (virtual rows kb * I + i, fixed-order block reduction),
+    forced at small sizes by shrinking the block to 64 rows."""
+    monkeypatch.setenv("CSTF_L2_BLOCK_ROWS", "64")
+    dims = (90, 2000, 700, 40)
+    idx, vals = datagen.coo(dims, (2, 2, 3, 1), 120000, 21)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    gi, gv = X.export_coo()
+    assert np.array_equal(gv, ref.vals) and all(np.array_equal(a, b) for a, b in zip(gi, ref.idx))
+    F = datagen.init_factors(dims, R, 3)
+    Fd = [cu(f) for f in F]
+    for n in range(4):
+        M = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        assert normwise(host(M), oracle.mttkrp(ref, n, F)) <= TOL, n
+    lam = cu(np.zeros(R))
+    gpu = B.cstf_factorize(X, Fd, lam, B.make_opts(R, outer_iters=3, tol=1e-2))
+    orc = oracle.factorize(ref, F, outer_iters=3, tol=1e-2)
+    n_, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6

@@ -34,6 +34,7 @@ from paper_conf_icpp_sohksc24_b200 import costmodel as cm  # noqa: E402
 METRIC = "cSTF outer-iteration time (s) and ADMM update HBM GB/s at 1/2/4/8 B200"
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_TFLOPS = 37.1      # measured on this pool's B200 (DFMA and DMMA alike), profiles/r01_microbench.txt
+L2_GATHER_GBS = 19890.0      # measured L2->SM random 256-byte row gathers, 7.4 MB tables (same microbench)
 
 
 def load_peaks():
@@ -72,7 +73,7 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
         except Exception:
             self.proc = None
@@ -183,7 +184,7 @@ def config_dict(cfg):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="nell2", choices=sorted(datagen.CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -273,7 +274,16 @@ def main():
                 "algorithmic_bytes_per_launch": byts / launches_per,
                 "avg_launch_ms": mtt_ms / launches_per,
                 "per_mode_ms": (mp[:, 1] / K).tolist()}
+        # second view (not the contract's roofline): factor-row bytes the kernel gathers
+        # (N-1 rows of R doubles per nonzero) vs the measured L2->SM gather rate
+        gathered = nnz * (N - 1) * R * 8 * N
+        line_gather = {"bound": "l2_gather", "achieved": gathered / (mtt_ms * 1e-3) / 1e9,
+                       "peak": L2_GATHER_GBS, "unit": "GB/s",
+                       "frac": gathered / (mtt_ms * 1e-3) / 1e9 / L2_GATHER_GBS,
+                       "note": "gathered row bytes incl. L1 hits; meaningful when the factors are L2-resident",
+                       "peak_source": "tools/microbench.cu, profiles/r01_microbench.txt"}
     else:
+        line_gather = None
         fl = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
         ach = fl / (upd_ms * 1e-3) / 1e12
         roof = {"kernel": "admm (k_admm_dmma, row-resident)", "bound": "tensor", "achieved": ach,
@@ -286,7 +296,7 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (datagen recipe, shapes of PAPER.md Table 2)",
             "config": config_dict(cfg), "gpu_launches": int(launches),
-            "roofline": roof, "admm_update_gbs": admm_gbs,
+            "roofline": roof, "roofline_l2_gather": line_gather, "admm_update_gbs": admm_gbs,
             "phases_ms_per_step": phase_ms, "clocks": clk,
             "setup": {"generate_s": t_gen, "load_coo_s": t_load, "nnz_coalesced": nnz}}
     # end to end through the public API with HOST buffers (pinned), one outer iteration per step

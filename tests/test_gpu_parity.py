@@ -425,3 +425,72 @@ def test_mttkrp_l2_blocked_copies(B, R, monkeypatch):
     orc = oracle.factorize(ref, F, outer_iters=3, tol=1e-2)
     n_, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+
+
+def test_factorize_bitwise_deterministic(B):
+    """Fixed grids and fixed reduction orders everywhere: two runs are bit-identical."""
+    c = datagen.CONFIGS["enron"].scaled(60, nnz_factor=1000)
+    idx, vals = c.generate()
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    start = datagen.init_factors(c.dims, 16, 2)
+    outs = []
+    for _ in range(2):
+        F = [cu(f) for f in start]
+        lam = cu(np.zeros(16))
+        rep = B.cstf_factorize(X, F, lam, B.make_opts(16, outer_iters=4, tol=1e-2))
+        outs.append((rep["fit"].tobytes(), rep["iters"].tobytes(), b"".join(host(f).tobytes() for f in F)))
+    assert outs[0] == outs[1]
+
+
+def test_eight_mode_tensor(B):
+    """N = 8 (7 other modes: 48-byte records, generic MTTKRP path) end to end."""
+    dims = (5, 4, 6, 3, 7, 4, 5, 3)
+    idx, vals = datagen.coo(dims, (1, 2, 1, 1, 2, 1, 1, 1), 4000, 31)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    assert X.info()["hash"] == ref.hash
+    R = 4
+    F = datagen.init_factors(dims, R, 5)
+    for n in (0, 7):
+        M = cu(np.zeros((dims[n], R)))
+        B.cstf_mttkrp(X, n, [cu(f) for f in F], M)
+        assert normwise(host(M), oracle.mttkrp(ref, n, F)) <= TOL
+    Fd = [cu(f) for f in F]
+    lam = cu(np.zeros(R))
+    gpu = B.cstf_factorize(X, Fd, lam, B.make_opts(R, outer_iters=3, tol=1e-2))
+    orc = oracle.factorize(ref, F, outer_iters=3, tol=1e-2)
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+
+
+def test_dead_column_and_rank_one(B):
+    """A component that dies (zero column, lambda = 0, reading D8) stays zero without NaN;
+    R = 1 runs the generic widths."""
+    c = datagen.CONFIGS["nell2"].scaled(100, nnz_factor=5000)
+    idx, vals = c.generate()
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    ref = oracle.coalesce(c.dims, idx, vals)
+    for R in (1, 6):
+        F = datagen.init_factors(c.dims, R, 8)
+        if R > 1:
+            for f in F:
+                f[:, 2] = 0.0                      # component 2 is dead from the start
+        Fd = [cu(f) for f in F]
+        lam = cu(np.zeros(R))
+        gpu = B.cstf_factorize(X, Fd, lam, B.make_opts(R, outer_iters=3, tol=1e-2))
+        orc = oracle.factorize(ref, F, outer_iters=3, tol=1e-2)
+        assert np.all(np.isfinite(gpu["fit"]))
+        assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+        if R > 1:
+            assert host(lam)[2] == 0.0 and all(np.all(host(f)[:, 2] == 0.0) for f in Fd)
+
+
+def test_nonfinite_input_is_reported(B):
+    dims = (20, 15, 10)
+    idx, vals = datagen.coo(dims, (1, 1, 1), 500, 4)
+    vals = vals.copy()
+    vals[7] = np.inf
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    F = [cu(f) for f in datagen.init_factors(dims, 4, 1)]
+    with pytest.raises(B.CstfError) as e:
+        B.cstf_factorize(X, F, cu(np.zeros(4)), B.make_opts(4, outer_iters=2, tol=1e-2))
+    assert e.value.status in (B.CSTF_ERR_NUMERIC, B.CSTF_ERR_NOT_SPD)

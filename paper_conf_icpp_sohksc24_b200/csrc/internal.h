@@ -118,6 +118,9 @@ struct ModeStore {
   mutable DevBuf wstart;    // int64[nwchunks+1]
   mutable DevBuf ckb;       // int32[nctachunks]
   mutable int64_t nwchunks = 0, nctachunks = 0;
+  // cached chunk boundaries of the MTTKRP work split (depend only on the store)
+  mutable DevBuf clb, ccont;
+  mutable int64_t cchunk = -1, cnchunks = 0;
 };
 inline int record_bytes(int N) { return ((4 * (N - 1) + 8) + 15) / 16 * 16; }
 

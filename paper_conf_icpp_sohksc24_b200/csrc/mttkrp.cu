@@ -277,32 +277,37 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
   }
 }
 
-// Add the carries of every row that continues across chunks, in chunk order.
-// The run of carry chunks of row h ends at the chunk holding h's last nonzero
-// (known from rowptr), so the loop has a known trip count and its loads pipeline.
-__global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks, const int64_t* __restrict__ rowptr,
-                              int64_t chunk, const int64_t* __restrict__ wstart,
-                              const double* __restrict__ carry, int R, double* __restrict__ M) {
+// Carry fix-up.  The run of carry chunks of row h is [c0, cend]: c0 = the chunk
+// after h's owner, cend = the chunk holding h's last nonzero.  Two levels in a
+// fixed order (deterministic): groups of kFixGroup consecutive carries aligned
+// at c0 are summed by one warp each, then the group sums of a run are added in
+// order to M[h].  Heavy power-law rows (hundreds of carries) are thus spread
+// over many warps instead of one.
+constexpr int kFixGroup = 16;
+
+__device__ __forceinline__ int64_t chunk_of(int64_t p, int64_t chunk, const int64_t* wstart, int64_t nchunks) {
+  if (!wstart) return p / chunk;
+  int64_t lo = 0, hi = nchunks - 1;            // last chunk with wstart <= p
+  while (lo < hi) {
+    const int64_t mid = (lo + hi + 1) >> 1;
+    if (wstart[mid] <= p) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__global__ void k_carry_groups(const int32_t* __restrict__ cont, int64_t nchunks, const int64_t* __restrict__ rowptr,
+                               int64_t chunk, const int64_t* __restrict__ wstart,
+                               const double* __restrict__ carry, int R, double* __restrict__ gsum) {
   const int lane = threadIdx.x & 31;
   const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t c = warp0; c < nchunks; c += nwarps) {
     const int32_t h = cont[c];
-    if (h < 0 || (c > 0 && cont[c - 1] == h)) continue;
-    const int64_t plast = rowptr[h + 1] - 1;           // last nonzero of row h
-    int64_t cend;                                      // chunk holding plast
-    if (!wstart) {
-      cend = plast / chunk;
-    } else {
-      int64_t lo = c, hi = nchunks - 1;                // last chunk with wstart <= plast
-      while (lo < hi) {
-        const int64_t mid = (lo + hi + 1) >> 1;
-        if (wstart[mid] <= plast) lo = mid; else hi = mid - 1;
-      }
-      cend = lo;
-    }
+    if (h < 0) continue;
+    const int64_t c0 = chunk_of(rowptr[h], chunk, wstart, nchunks) + 1;
+    if ((c - c0) % kFixGroup != 0) continue;                // not a group leader
+    const int64_t cend = min(chunk_of(rowptr[h + 1] - 1, chunk, wstart, nchunks), c + kFixGroup - 1);
     for (int col = lane; col < R; col += 32) {
-      // four interleaved partial sums (fixed combination order) keep 16 loads in flight
       double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
       int64_t cc = c;
       for (; cc + 3 <= cend; cc += 4) {
@@ -312,7 +317,25 @@ __global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks,
         s3 += carry[(cc + 3) * R + col];
       }
       for (; cc <= cend; cc++) s0 += carry[cc * R + col];
-      M[(int64_t)h * R + col] += (s0 + s1) + (s2 + s3);
+      gsum[c * R + col] = (s0 + s1) + (s2 + s3);
+    }
+  }
+}
+
+__global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks, const int64_t* __restrict__ rowptr,
+                              int64_t chunk, const int64_t* __restrict__ wstart,
+                              const double* __restrict__ gsum, int R, double* __restrict__ M) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t c = warp0; c < nchunks; c += nwarps) {
+    const int32_t h = cont[c];
+    if (h < 0 || (c > 0 && cont[c - 1] == h)) continue;     // run starts only
+    const int64_t cend = chunk_of(rowptr[h + 1] - 1, chunk, wstart, nchunks);
+    for (int col = lane; col < R; col += 32) {
+      double s = 0.0;
+      for (int64_t cc = c; cc <= cend; cc += kFixGroup) s += gsum[cc * R + col];
+      M[(int64_t)h * R + col] += s;
     }
   }
 }
@@ -391,7 +414,7 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st) {
 }
 
 struct Workspace {
-  DevBuf lb, cont, carry, partial, kbptr;
+  DevBuf lb, cont, carry, gsum, partial, kbptr;
   std::vector<int64_t> hk;
 };
 
@@ -472,9 +495,13 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     if (chunk > 8192) chunk = 8192;
     nchunks = nnz > 0 ? (nnz + chunk - 1) / chunk : 1;
   }
-  CSTF_TRY(w.lb.ensure((size_t)(nchunks + 1) * 8));
-  CSTF_TRY(w.cont.ensure((size_t)nchunks * 4));
   CSTF_TRY(w.carry.ensure((size_t)nchunks * R * 8));
+  CSTF_TRY(w.gsum.ensure((size_t)nchunks * R * 8));
+  const bool fresh = ms.cchunk != chunk || ms.cnchunks != nchunks;   // boundaries cached per mode
+  if (fresh) {
+    CSTF_TRY(ms.clb.alloc((size_t)(nchunks + 1) * 8));
+    CSTF_TRY(ms.ccont.alloc((size_t)nchunks * 4));
+  }
   double* out = d_M;
   if (ms.tiled) {
     CSTF_TRY(w.partial.ensure((size_t)ms.Ivirt * R * 8));
@@ -491,18 +518,20 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.chunk = chunk;
   a.nchunks = nchunks;
   a.R = R;
-  a.lb = w.lb.as<int64_t>();
-  a.cont = w.cont.as<int32_t>();
+  a.lb = ms.clb.as<int64_t>();
+  a.cont = ms.ccont.as<int32_t>();
   a.M = out;
   a.carry = w.carry.as<double>();
   if (ms.I == 0) return CSTF_OK;
   int64_t nl = 0;
-  {
+  if (fresh) {
     const int g = (int)std::min<int64_t>((nchunks + 1 + 255) / 256, (int64_t)di.sms * 8);
-    k_chunk_bounds<<<g, 256, 0, st>>>(a.rowptr, ms.Ivirt, nnz, chunk, nchunks, a.wstart, w.lb.as<int64_t>(),
-                                       w.cont.as<int32_t>());
+    k_chunk_bounds<<<g, 256, 0, st>>>(a.rowptr, ms.Ivirt, nnz, chunk, nchunks, a.wstart, ms.clb.as<int64_t>(),
+                                       ms.ccont.as<int32_t>());
     CSTF_LAUNCHED();
     nl++;
+    ms.cchunk = chunk;
+    ms.cnchunks = nchunks;
   }
   const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
   const int tgrid = (int)std::min<int64_t>(std::max<int64_t>(ms.nctachunks, 1), (int64_t)di.sms * 2);
@@ -511,9 +540,11 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   nl++;
   if (nchunks > 1) {
     const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);
-    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, a.carry, R, out);
+    k_carry_groups<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, a.carry, R, w.gsum.as<double>());
     CSTF_LAUNCHED();
-    nl++;
+    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, w.gsum.as<double>(), R, out);
+    CSTF_LAUNCHED();
+    nl += 2;
   }
   if (ms.tiled) {
     const int64_t n = ms.I * R;

@@ -184,7 +184,7 @@ def config_dict(cfg):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="nell2", choices=sorted(datagen.CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
@@ -226,15 +226,17 @@ def main():
     def opts(n, timing=False):
         return B.make_opts(R, outer_iters=n, tol=0.0, max_iter=10, timing=timing)
 
+    # nvidia-smi needs a few hundred ms before its first sample: start it now, so
+    # it samples the (identical) warm-up work and the timed region
+    clocks = ClockSampler(local)
+    clocks.start()
     # warm-up: W outer iterations
     B.cstf_factorize(X, F, lam, opts(max(args.warmup, 3)), comm=comm)
     torch.cuda.synchronize()
     # timed: K outer iterations in one call (each call starts with the init pass: included)
-    clocks = ClockSampler(local)
     if dist:
         dist.barrier()
     torch.cuda.synchronize()
-    clocks.start()
     l0 = B.cstf_kernel_launch_count()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)

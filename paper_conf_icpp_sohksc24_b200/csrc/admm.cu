@@ -54,6 +54,8 @@ struct KArgs {
   int sums_from;           // first local pass whose residual sums are formed
   double* slots;           // [kiters][gridDim][4]
   double* gpart;           // optional: per-CTA Gram partials [grid][NT(NT+1)/2][64]
+  double* peer[7];         // optional: the same rows of the factor replicas of the other ranks
+  int npeer;               //   (CUDA-IPC / NVLink peer memory): fused all-gather (f4)
 };
 
 // Alg. 2 l.7: argmin_h r(h) + rho/2 (h - x)^2 for the element-wise regularisers
@@ -226,14 +228,21 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
         if (full) {
           __stcs(reinterpret_cast<double2*>(a.Hout + base + col), make_double2(h[t][0], h[t][1]));
           if (!MU) __stcs(reinterpret_cast<double2*>(a.Uout + base + col), make_double2(u[t][0], u[t][1]));
+          for (int p = 0; p < a.npeer; p++)     // the row lands in every replica (peer stores)
+            *reinterpret_cast<double2*>(a.peer[p] + base + col) = make_double2(h[t][0], h[t][1]);
         } else {
 #pragma unroll
           for (int i = 0; i < 2; i++)
-            if (col + i < R) { a.Hout[base + col + i] = h[t][i]; if (!MU) a.Uout[base + col + i] = u[t][i]; }
+            if (col + i < R) {
+              a.Hout[base + col + i] = h[t][i];
+              if (!MU) a.Uout[base + col + i] = u[t][i];
+              for (int p = 0; p < a.npeer; p++) a.peer[p][base + col + i] = h[t][i];
+            }
         }
       }
     }
   }
+  if (a.npeer) __threadfence_system();     // peer stores visible before the kernel completes
   __syncthreads();
   // fixed-order CTA reduction of the per-thread slots
   for (int x = tid; x < nsl * 4; x += kThreads) {
@@ -619,6 +628,7 @@ cstf_status mu_run(const UpdArgs& A, cudaStream_t st) {
   const bool gram = A.G != nullptr && A.R <= 32;
   if (gram) CSTF_TRY(w.gpart.ensure((size_t)maxgrid * 10 * 64 * 8));
   KArgs k{};
+  k.npeer = 0;
   k.M = A.M; k.H = A.H; k.U = nullptr; k.Hout = A.H; k.Uout = nullptr;
   k.hscale = A.hscale; k.mscale = A.mscale; k.I = A.I; k.R = A.R; k.inv = A.S; k.scal = A.scal;
   k.flag = A.flag; k.prox = 0; k.alpha = 0.0; k.slots = w.slots.as<double>();
@@ -685,6 +695,8 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
   k.alpha = A.alpha;
   k.slots = w.slots.as<double>();
   k.gpart = nullptr;
+  k.npeer = 0;
+  A.peer_done = false;
   if (spec) {
     for (int b = 0; b < 2; b++) {
       CSTF_TRY(w.hs[b].ensure((size_t)I * R * 8));
@@ -706,6 +718,10 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
     k.sums_from = spec ? 0 : (last ? kk - 1 : kk);
     const bool gram_now = fuse_gram && last;
     k.gpart = gram_now ? w.gpart.as<double>() : nullptr;
+    // fused all-gather (f4): only the final in-place chunk of the fixed-iteration path
+    k.npeer = (!spec && last && A.npeer > 0) ? A.npeer : 0;
+    for (int p = 0; p < k.npeer; p++) k.peer[p] = A.peerH[p];
+    if (k.npeer) A.peer_done = true;
     if (spec && kchunk > 1) {
       k.Hout = w.hs[pp].as<double>();
       k.Uout = w.us[pp].as<double>();
@@ -771,6 +787,7 @@ cstf_status admm_run(const AdmmArgs& A, const cstf_comm* comm, cudaStream_t st,
         k.kiters = dj - j0;
         k.sums_from = k.kiters;  // sums already known
         k.gpart = nullptr;
+        k.npeer = 0;
         k.Hout = A.H; k.Uout = A.U;
         CSTF_TRY(launch_kernel(k, grid, false, st));
         nl++;

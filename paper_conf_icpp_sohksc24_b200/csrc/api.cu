@@ -1,4 +1,5 @@
 // extern "C" entry points of libcstf (include/cstf.h) and the Alg. 1 driver.
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -36,6 +37,12 @@ bool rank_ok(int R) { return R >= 1 && R <= 128; }
 // Device-side scratch of one factorize / admm_update call, cached per device.
 struct DriverWs {
   DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8], S;
+  // distributed: all internal factor replicas in one allocation, mapped by the
+  // other ranks through CUDA IPC (NVLink peer memory) for the fused all-gather
+  DevBuf facall, xchg;
+  void* ipc_for = nullptr;
+  const cstf_comm* ipc_comm = nullptr;
+  double* ipc_peer[8] = {nullptr};
   double* host_small = nullptr;  // pinned: fit, flags
   cudaStream_t side = nullptr;   // the R x R step of a mode overlaps its MTTKRP
   cudaEvent_t fork = nullptr, join = nullptr;
@@ -52,6 +59,53 @@ DriverWs& dws() {
     cudaEventCreateWithFlags(&r.join, cudaEventDisableTiming);
   }
   return r;
+}
+
+// Map every other rank's factor replicas (CUDA IPC handles exchanged through the
+// communicator).  Collective; returns false on every rank if any rank fails.
+bool open_peers(DriverWs& w, const cstf_comm* comm, cudaStream_t st) {
+  const int P = comm_nranks(comm), me = comm_rank(comm);
+  if (w.ipc_for == w.facall.p && w.ipc_comm == comm) return true;
+  for (int r = 0; r < 8; r++)
+    if (w.ipc_peer[r]) { cudaIpcCloseMemHandle(w.ipc_peer[r]); w.ipc_peer[r] = nullptr; }
+  w.ipc_for = nullptr;
+  const char* env = getenv("CSTF_PEER_STORE");
+  double ok = (P <= 8 && !(env && atoi(env) == 0)) ? 1.0 : 0.0;
+  cudaIpcMemHandle_t h;
+  memset(&h, 0, sizeof(h));
+  if (ok > 0 && cudaIpcGetMemHandle(&h, w.facall.p) != cudaSuccess) { cudaGetLastError(); ok = 0; }
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+  if (w.xchg.ensure((size_t)(8 * P + 8) * 8) != CSTF_OK) return false;
+  double* d = w.xchg.as<double>();
+  if (cudaMemcpyAsync(d + 8 * P, &h, 64, cudaMemcpyHostToDevice, st) != cudaSuccess) return false;
+  if (comm_allgather_f64(comm, d + 8 * P, d, 8, st) != CSTF_OK) return false;
+  std::vector<cudaIpcMemHandle_t> hs((size_t)P);
+  if (cudaMemcpyAsync(hs.data(), d, (size_t)P * 64, cudaMemcpyDeviceToHost, st) != cudaSuccess) return false;
+  if (cudaStreamSynchronize(st) != cudaSuccess) return false;
+  for (int r = 0; r < P && ok > 0; r++) {
+    if (r == me) continue;
+    void* ptr = nullptr;
+    if (cudaIpcOpenMemHandle(&ptr, hs[(size_t)r], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+      cudaGetLastError();
+      ok = 0;
+    } else {
+      w.ipc_peer[r] = static_cast<double*>(ptr);
+    }
+  }
+  // consensus: every rank uses peer stores or none does
+  double fails = ok > 0 ? 0.0 : 1.0;
+  if (cudaMemcpyAsync(d, &fails, 8, cudaMemcpyHostToDevice, st) != cudaSuccess) return false;
+  if (comm_allreduce_f64(comm, d, 1, st) != CSTF_OK) return false;
+  if (cudaMemcpyAsync(&fails, d, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) return false;
+  if (cudaStreamSynchronize(st) != cudaSuccess) return false;
+  if (fails > 0) {
+    for (int r = 0; r < 8; r++)
+      if (w.ipc_peer[r]) { cudaIpcCloseMemHandle(w.ipc_peer[r]); w.ipc_peer[r] = nullptr; }
+    return false;
+  }
+  w.ipc_for = w.facall.p;
+  w.ipc_comm = comm;
+  return true;
 }
 
 cstf_status check_flag(const int* d_flag, cudaStream_t st) {
@@ -124,15 +178,22 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   // internal (relabelled, zero-padded) row order; its own rows are the slice
   // [rank*B_n, (rank+1)*B_n).  Single GPU: the caller's buffers, all rows local.
   std::vector<double*> fac(N);
-  std::vector<int64_t> Ifull(N), Iloc(N), off(N);
+  std::vector<int64_t> Ifull(N), Iloc(N), off(N), facoff(N);
+  if (dist) {                         // one allocation for all replicas (IPC-mappable)
+    int64_t tot = 0;
+    for (int n = 0; n < N; n++) {
+      facoff[n] = tot;
+      tot += ((int64_t)X->nranks * X->rows_per_rank[n] * R + 31) / 32 * 32;
+    }
+    CSTF_TRY(w.facall.ensure((size_t)tot * 8));
+  }
   for (int n = 0; n < N; n++) {
     if (dist) {
       const int64_t B = X->rows_per_rank[n];
       Ifull[n] = (int64_t)X->nranks * B;
       Iloc[n] = B;
       off[n] = (int64_t)X->rank * B * R;
-      CSTF_TRY(w.Fi[n].ensure((size_t)Ifull[n] * R * 8));
-      fac[n] = w.Fi[n].as<double>();
+      fac[n] = w.facall.as<double>() + facoff[n];
       CSTF_CUDA(cudaMemsetAsync(fac[n], 0, (size_t)Ifull[n] * R * 8, st));
       CSTF_TRY(relabel_rows(d_factors[n], X->relabel[n].as<int32_t>(), X->dims[n], R, fac[n], 1, st));
     } else {
@@ -143,6 +204,9 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   }
   int64_t Imax = 0, Usum = 0;
   for (int n = 0; n < N; n++) { Imax = std::max(Imax, Iloc[n]); Usum += Iloc[n] * R; }
+  // f4: fused all-gather through peer stores from the ADMM epilogue (falls back to
+  // the NCCL / host all-gather when IPC mapping is unavailable or disabled)
+  const bool peers = dist && open_peers(w, comm, st);
   CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
   CSTF_TRY(w.lam.ensure((size_t)N * R * 8));
   CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
@@ -169,6 +233,9 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     CSTF_TRY(gram_raw(fac[n], Ifull[n], R, Gn, st));
     if (o->normalize_init) CSTF_TRY(normalize_from_gram(fac[n], Ifull[n], R, Gn, lam + n * R, st));
     CSTF_TRY(fill(lam + n * R, R, 1.0, st));
+  }
+  if (peers) {   // no rank may peer-store into a replica another rank is still initialising / reading
+    CSTF_TRY(comm_allreduce_f64(comm, w.xchg.as<double>(), 1, st));
   }
   PhaseTimer tm;
   tm.on = o->timing != 0;
@@ -222,6 +289,14 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       if (o->update == CSTF_UPDATE_ADMM) {
         fused = admm_can_fuse_gram(R, o->admm.tol);
         a.G = fused ? Gn : nullptr;      // a7 fused into the ADMM epilogue
+        double* peerH[8];
+        if (peers) {                     // f4: this rank's rows go straight into every replica
+          int np = 0;
+          for (int r = 0; r < X->nranks; r++)
+            if (r != X->rank) peerH[np++] = w.ipc_peer[r] + facoff[n] + off[n];
+          a.peerH = peerH;
+          a.npeer = np;
+        }
         CSTF_TRY(admm_run(a, comm, st, nullptr, &iters, nullptr));
       } else {                           // f1: HALS / MU on the same M, S
         UpdArgs u;
@@ -244,11 +319,14 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
         CSTF_TRY(gram_raw(Hn, I, R, Gn, st));
         tm.end(n, CSTF_PHASE_GRAM);
       }
-      if (dist) {                        // every rank needs the updated factor for the next MTTKRPs
+      if (dist && !a.peer_done) {        // every rank needs the updated factor for the next MTTKRPs
         tm.begin(n, CSTF_PHASE_COMM);
         CSTF_TRY(comm_allgather_f64(comm, Hn, fac[n], (size_t)I * R, st));
         tm.end(n, CSTF_PHASE_COMM);
       }
+      // (with peer stores, the all-reduce of the Gram below is the barrier after
+      // which every replica holds every rank's rows: each rank joins it only after
+      // its ADMM kernel -- which ends with a system-scope fence -- has completed)
       tm.begin(n, CSTF_PHASE_NORMALIZE);
       CSTF_TRY(comm_allreduce_f64(comm, Gn, (size_t)R * R, st));
       CSTF_TRY(gram_to_lambda(Gn, R, lam + n * R, st));

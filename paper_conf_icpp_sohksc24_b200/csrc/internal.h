@@ -207,6 +207,9 @@ struct AdmmArgs {
   int prox;
   int variant;
   double alpha = 0.0;    // L1 weight (prox 2/3)
+  double* const* peerH = nullptr;  // fused all-gather: this rank's rows in each peer replica
+  int npeer = 0;
+  mutable bool peer_done = false;  // out: the rows were stored into the peers
 };
 cstf_status admm_run(const AdmmArgs& a, const cstf_comm* comm, cudaStream_t st,
                      cstf_admm_stats* stats, int* iters_out, int64_t* launches);

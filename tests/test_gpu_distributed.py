@@ -29,9 +29,12 @@ X = B.cstf_tensor_load_coo(c.dims, idx, vals, comm=comm)
 start = datagen.init_factors(c.dims, R, c.seed)
 F = [torch.from_numpy(f.copy()).cuda() for f in start]
 lam = torch.zeros(R, dtype=torch.float64, device="cuda")
-rep = B.cstf_factorize(X, F, lam, B.make_opts(R, outer_iters=outer, tol=tol, max_iter=10), comm=comm)
+rep = B.cstf_factorize(X, F, lam, B.make_opts(R, outer_iters=outer, tol=tol, max_iter=10, timing=True), comm=comm)
+rep2 = B.cstf_factorize(X, [torch.from_numpy(f.copy()).cuda() for f in start], lam.clone(),
+                        B.make_opts(R, outer_iters=outer, tol=tol, max_iter=10), comm=comm)   # back-to-back calls
 torch.cuda.synchronize()
-out = {"fit": rep["fit"].tolist(), "iters": rep["iters"].tolist()}
+assert np.array_equal(rep["fit"], rep2["fit"]), (rep["fit"], rep2["fit"])
+out = {"fit": rep["fit"].tolist(), "iters": rep["iters"].tolist(), "comm_ms": rep["phase_ms"]["COMM"]}
 if rank == 0:
     ref = oracle.coalesce(c.dims, idx, vals)
     orc = oracle.factorize(ref, start, outer_iters=outer, tol=tol, max_iter=10)
@@ -64,16 +67,21 @@ def run(tmp_path, nproc, case, port):
     return res
 
 
-@pytest.mark.parametrize("nproc,case,port", [
-    (2, ("nell2", 40, 16, 1e-2, 5), 29611),
-    (3, ("enron", 60, 8, 1e-2, 5), 29612),
-    (2, ("delicious", 2000, 32, 0.0, 3), 29613),
+@pytest.mark.parametrize("nproc,case,port,peer", [
+    (2, ("nell2", 40, 16, 1e-2, 5), 29611, "1"),
+    (3, ("enron", 60, 8, 1e-2, 5), 29612, "1"),
+    (2, ("delicious", 2000, 32, 0.0, 3), 29613, "1"),     # eps = 0: ADMM epilogue peer stores (f4)
+    (3, ("nell2", 40, 32, 0.0, 4), 29614, "1"),
+    (3, ("nell2", 40, 32, 0.0, 4), 29615, "0"),           # same case through the plain all-gather
 ])
-def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port):
+def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port, peer, monkeypatch):
+    monkeypatch.setenv("CSTF_PEER_STORE", peer)
     res = run(tmp_path, nproc, case, port)
     r0 = res[0]
     for rk in range(1, nproc):          # every rank took the same decisions
         assert res[rk]["fit"] == r0["fit"] and res[rk]["iters"] == r0["iters"]
     assert r0["fit_rel"] <= 1e-6
+    if peer == "1" and case[3] == 0.0 and case[2] <= 32:
+        assert r0["comm_ms"] == 0.0          # no separate all-gather ran: rows were peer-stored
     if not r0["tie"]:
         assert r0["fac_rel"] <= 1e-6 and r0["lam_rel"] <= 1e-6

@@ -147,9 +147,14 @@ __global__ void k_gram_normalize(double* __restrict__ G, int R, double* __restri
 __global__ void k_scale_cols(double* __restrict__ H, int64_t I, int R, const double* __restrict__ lam,
                              int divide) {
   const int64_t n = I * R;
-  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
-       x += (int64_t)gridDim.x * blockDim.x) {
-    const double l = lam[x % R];
+  const int64_t x0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int64_t step = (int64_t)gridDim.x * blockDim.x;
+  const int dstep = (int)(step % R);          // column advances by a constant: no per-element modulo
+  int col = (int)(x0 % R);
+  for (int64_t x = x0; x < n; x += step) {
+    const double l = lam[col];
+    col += dstep;
+    if (col >= R) col -= R;
     if (divide) {
       if (l > 0.0) H[x] = H[x] / l;
     } else {
@@ -280,9 +285,15 @@ __global__ void __launch_bounds__(256) k_fit_partial(const double* __restrict__ 
   __shared__ double sh[256];
   const int64_t n = I * R;
   double acc = 0.0;
-  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
-       x += (int64_t)gridDim.x * blockDim.x)
-    acc = fma(M[x] * H[x], colw[x % R], acc);
+  const int64_t x0 = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+  const int64_t step = (int64_t)gridDim.x * blockDim.x;
+  const int dstep = (int)(step % R);
+  int col = (int)(x0 % R);
+  for (int64_t x = x0; x < n; x += step) {
+    acc = fma(M[x] * H[x], colw[col], acc);
+    col += dstep;
+    if (col >= R) col -= R;
+  }
   sh[threadIdx.x] = acc;
   __syncthreads();
   for (int s = 128; s > 0; s >>= 1) {

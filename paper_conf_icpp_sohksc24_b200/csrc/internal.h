@@ -61,16 +61,6 @@ struct DevBuf {
   template <class T> T* as() const { return static_cast<T*>(p); }
 };
 
-// Grow-only scratch arena carved into aligned slices.
-struct Arena {
-  DevBuf buf;
-  size_t used = 0;
-  std::vector<size_t> pending;  // requested sizes while planning
-  void reset() { used = 0; }
-  // returns aligned pointer inside buf (caller must have ensured capacity)
-  void* take(size_t n);
-};
-
 // ---------------------------------------------------------------- comm
 struct Comm {
   int nranks = 1;

@@ -66,12 +66,6 @@ cstf_status DevBuf::ensure(size_t n) {
   return alloc(n);
 }
 
-void* Arena::take(size_t n) {
-  size_t off = (used + 255) & ~(size_t)255;
-  used = off + n;
-  return static_cast<char*>(buf.p) + off;
-}
-
 // ------------------------------------------------------------------ NCCL (dlopen)
 namespace {
 struct NcclApi {

@@ -35,6 +35,8 @@ METRIC = "cSTF outer-iteration time (s) and ADMM update HBM GB/s at 1/2/4/8 B200
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FP64_PEAK_TFLOPS = 37.1      # measured on this pool's B200 (DFMA and DMMA alike), profiles/r01_microbench.txt
 L2_GATHER_GBS = 19890.0      # measured L2->SM random 256-byte row gathers, 7.4 MB tables (same microbench)
+L1_GATHER_GBS = 28855.0      # measured all-L1-hit 256-byte row gathers (16 lanes x 16 B, two 200-row tables):
+                             # the on-chip ceiling of the MTTKRP access (tools/gather_probe.cu, profiles/r01_gather_probe.txt)
 
 
 def load_peaks():
@@ -277,16 +279,28 @@ def main():
                 "avg_launch_ms": mtt_ms / launches_per,
                 "per_mode_ms": (mp[:, 1] / K).tolist()}
         # second view (not the contract's roofline): factor-row bytes the kernel gathers
-        # (N-1 rows of R doubles per nonzero) vs the measured L2->SM gather rate
+        # (N-1 rows of R doubles per nonzero) vs the measured all-L1-hit gather ceiling
         gathered = nnz * (N - 1) * R * 8 * N
-        line_gather = {"bound": "l2_gather", "achieved": gathered / (mtt_ms * 1e-3) / 1e9,
-                       "peak": L2_GATHER_GBS, "unit": "GB/s",
-                       "frac": gathered / (mtt_ms * 1e-3) / 1e9 / L2_GATHER_GBS,
-                       "note": "gathered row bytes incl. L1 hits; meaningful when the factors are L2-resident",
-                       "peak_source": "tools/microbench.cu, profiles/r01_microbench.txt"}
+        line_gather = {"bound": "onchip_gather", "achieved": gathered / (mtt_ms * 1e-3) / 1e9,
+                       "peak": L1_GATHER_GBS, "unit": "GB/s",
+                       "frac": gathered / (mtt_ms * 1e-3) / 1e9 / L1_GATHER_GBS,
+                       "l2_gather_peak": L2_GATHER_GBS,
+                       "note": "factor-row bytes moved into registers (N-1 rows of R doubles per nonzero, "
+                               "L1 hits included) vs the all-L1-hit gather ceiling; meaningful when the "
+                               "factors are L2-resident",
+                       "peak_source": "tools/gather_probe.cu, profiles/r01_gather_probe.txt"}
     else:
         line_gather = None
-        fl = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
+    # the ADMM update (the paper's cuADMM) against the FP64 datapath, always reported
+    fl_admm = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
+    roof_admm = {"kernel": "admm (k_admm_dmma, row-resident)", "bound": "fp64",
+                 "achieved": fl_admm / (upd_ms * 1e-3) / 1e12 if upd_ms > 0 else None,
+                 "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
+                 "frac": fl_admm / (upd_ms * 1e-3) / 1e12 / FP64_PEAK_TFLOPS if upd_ms > 0 else None,
+                 "note": "DMMA and DFMA share one FP64 datapath on B200 (profiles/r01_fp64_probe.txt); "
+                         "flops = (2R^2 + 19R) I per inner iteration (Eq. 3), 10 iterations per mode"}
+    if mtt_ms < upd_ms:
+        fl = fl_admm
         ach = fl / (upd_ms * 1e-3) / 1e12
         roof = {"kernel": "admm (k_admm_dmma, row-resident)", "bound": "tensor", "achieved": ach,
                 "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS,
@@ -298,7 +312,7 @@ def main():
             "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (datagen recipe, shapes of PAPER.md Table 2)",
             "config": config_dict(cfg), "gpu_launches": int(launches),
-            "roofline": roof, "roofline_l2_gather": line_gather, "admm_update_gbs": admm_gbs,
+            "roofline": roof, "roofline_gather": line_gather, "roofline_admm": roof_admm, "admm_update_gbs": admm_gbs,
             "phases_ms_per_step": phase_ms, "clocks": clk,
             "setup": {"generate_s": t_gen, "load_coo_s": t_load, "nnz_coalesced": nnz}}
     # end to end through the public API with HOST buffers (pinned), one outer iteration per step

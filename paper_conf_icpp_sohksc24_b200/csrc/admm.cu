@@ -26,6 +26,8 @@
 //    registers) by 2 * NT(NT+1)/2 more DMMAs per 8 rows (Alg. 1 l.12 fused,
 //    R <= 32), and a per-column scale of M on load (lazy normalisation:
 //    M = M' diag(mscale)).
+#include <cstdlib>
+
 #include "internal.h"
 
 namespace cstf {
@@ -77,8 +79,9 @@ __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b)
 // RP = padded rank (multiple of 8, <= 64).  GRAM: fused Gram epilogue (RP <= 32).
 // MU: multiplicative update (f1, reading D22) in the same shape: A operand = h,
 // B = S (passed in a.inv), epilogue h <- h * m / (hS + 1e-16); no dual, no sums.
-template <int RP, bool GRAM, bool MU = false>
-__global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
+// IREG: Inv fragments held in registers (RP <= 32, 3 CTAs/SM) instead of read from SMEM per DMMA.
+template <int RP, bool GRAM, bool MU = false, bool IREG = false>
+__global__ void __launch_bounds__(kThreads, IREG ? 3 : 0) k_admm_dmma(KArgs a) {
   constexpr int NT = RP / 8;       // n-tiles of 8 columns
   constexpr int NC = 2 * NT;       // k-chunks of 4
   constexpr int NP = NT * (NT + 1) / 2;   // Gram tile pairs (a <= b)
@@ -105,9 +108,17 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
     sinv[x] = (k < R && n < R) ? a.inv[k * R + n] : 0.0;
   }
   __syncthreads();
-  double hs[NT][2], ms[NT][2];
+  double binv[IREG ? NC : 1][IREG ? NT : 1];
+  if constexpr (IREG) {
 #pragma unroll
-  for (int t = 0; t < NT; t++)
+    for (int c = 0; c < NC; c++)
+#pragma unroll
+      for (int t = 0; t < NT; t++) binv[c][t] = sinv[(c * NT + t) * 32 + lane];
+  }
+  constexpr int NS = IREG ? 1 : NT;   // IREG: column scales re-read per row group (register budget)
+  double hs[NS][2], ms[NS][2];
+#pragma unroll
+  for (int t = 0; t < NS; t++)
 #pragma unroll
     for (int i = 0; i < 2; i++) {
       const int col = 8 * t + 2 * q + i;
@@ -145,8 +156,14 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
       }
 #pragma unroll
       for (int i = 0; i < 2; i++) {
-        h[t][i] = h[t][i] * hs[t][i];
-        m[t][i] = m[t][i] * ms[t][i];
+        if constexpr (IREG) {
+          const int cc = 8 * t + 2 * q + i;
+          if (a.hscale && cc < R) h[t][i] = h[t][i] * __ldg(a.hscale + cc);
+          if (a.mscale && cc < R) m[t][i] = m[t][i] * __ldg(a.mscale + cc);
+        } else {
+          h[t][i] = h[t][i] * hs[t][i];
+          m[t][i] = m[t][i] * ms[t][i];
+        }
       }
     }
     for (int j = 0; j < kiters; j++) {
@@ -158,7 +175,10 @@ __global__ void __launch_bounds__(kThreads) k_admm_dmma(KArgs a) {
         const int tt = c >> 1, ii = c & 1;
         const double av = MU ? h[tt][ii] : fma(rho, h[tt][ii] + u[tt][ii], m[tt][ii]);   // M + rho (H + U)
 #pragma unroll
-        for (int t = 0; t < NT; t++) dmma(d[t][0], d[t][1], av, sinv[(c * NT + t) * 32 + lane]);
+        for (int t = 0; t < NT; t++) {
+          if constexpr (IREG) dmma(d[t][0], d[t][1], av, binv[c][t]);
+          else dmma(d[t][0], d[t][1], av, sinv[(c * NT + t) * 32 + lane]);
+        }
       }
       if (MU) {
 #pragma unroll
@@ -525,25 +545,34 @@ Workspace& ws() {
   return r;
 }
 
+// Register-resident Inv (3 CTAs/SM) for row-resident launches of several passes:
+// the DMMAs no longer wait on a shared-memory load each (Delicious mode 1, R = 32,
+// 10 passes: 15.3 -> 14.6 ms).  One-pass (streaming) launches are HBM-bound and
+// keep the 4-CTA/SM variant.  CSTF_ADMM_IREG=0/1 forces either (experiments).
+bool admm_ireg(int kiters) {
+  static const int v = [] { const char* e = getenv("CSTF_ADMM_IREG"); return e ? (e[0] == '1' ? 1 : 0) : -1; }();
+  return v < 0 ? kiters >= 4 : v == 1;
+}
+
 size_t dmma_smem(int RP, bool gram, int nsl) {
   const int NT = RP / 8;
   return (size_t)nsl * 4 * kThreads * 8 + (size_t)2 * NT * NT * 32 * 8 +
          (gram ? (size_t)kWarpsA * NT * (NT + 1) / 2 * 64 * 8 : 0);
 }
 
-template <int RP, bool GRAM, bool MU = false>
+template <int RP, bool GRAM, bool MU = false, bool IREG = false>
 cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
   const int nsl = k.kiters - k.sums_from;
   const size_t smem = dmma_smem(RP, GRAM, nsl);
   static int per_sm[kMaxK + 1] = {0};
   static bool attr = false;
   if (!attr) {
-    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM, MU>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM, MU, IREG>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)dmma_smem(RP, GRAM, kMaxK)));
     attr = true;
   }
   if (!per_sm[nsl]) {
-    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM, MU>, kThreads, smem));
+    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM, MU, IREG>, kThreads, smem));
     if (per_sm[nsl] < 1) per_sm[nsl] = 1;
   }
   const int64_t groups = (k.I + 7) / 8;
@@ -551,7 +580,7 @@ cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
   const int64_t cap = (int64_t)device_info().sms * per_sm[nsl];
   if (g > cap) g = cap;
   grid = (int)(g < 1 ? 1 : g);
-  k_admm_dmma<RP, GRAM, MU><<<grid, kThreads, smem, st>>>(k);
+  k_admm_dmma<RP, GRAM, MU, IREG><<<grid, kThreads, smem, st>>>(k);
   CSTF_LAUNCHED();
   return CSTF_OK;
 }
@@ -565,14 +594,18 @@ cstf_status launch_kernel(const KArgs& k, int& grid, bool gram, cudaStream_t st)
         case 8: return launch_dmma_t<8, true>(k, grid, st);
         case 16: return launch_dmma_t<16, true>(k, grid, st);
         case 24: return launch_dmma_t<24, true>(k, grid, st);
-        case 32: return launch_dmma_t<32, true>(k, grid, st);
+        case 32:
+          if (admm_ireg(k.kiters)) return launch_dmma_t<32, true, false, true>(k, grid, st);
+          return launch_dmma_t<32, true>(k, grid, st);
       }
     }
     switch (RP) {
       case 8: return launch_dmma_t<8, false>(k, grid, st);
       case 16: return launch_dmma_t<16, false>(k, grid, st);
       case 24: return launch_dmma_t<24, false>(k, grid, st);
-      case 32: return launch_dmma_t<32, false>(k, grid, st);
+      case 32:
+        if (admm_ireg(k.kiters)) return launch_dmma_t<32, false, false, true>(k, grid, st);
+        return launch_dmma_t<32, false>(k, grid, st);
       case 40: return launch_dmma_t<40, false>(k, grid, st);
       case 48: return launch_dmma_t<48, false>(k, grid, st);
       case 56: return launch_dmma_t<56, false>(k, grid, st);

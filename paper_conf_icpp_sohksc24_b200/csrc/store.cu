@@ -587,7 +587,10 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
       for (int q = N - 2; q >= 0 && !ms.tiled; q--) {     // largest other factor first
         const int tm = ms.other[q];
         const int64_t nb = (X->dims[tm] + l2rows - 1) / l2rows;
-        if (X->dims[tm] > 2 * l2rows && nb * ms.I <= ((int64_t)16 << 20) && nout >= 4 * nb * ms.I) {
+        static const int64_t maxv = getenv("CSTF_L2_BLOCK_MAXROWS") ? atoll(getenv("CSTF_L2_BLOCK_MAXROWS"))
+                                                                     : ((int64_t)16 << 20);
+        if (X->dims[tm] > 2 * l2rows && nb * ms.I <= maxv && nb * ms.I < ((int64_t)1 << 31) &&
+            nout >= 4 * nb * ms.I) {
           ms.tiled = true; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = q; t = tm;
         }
       }

@@ -18,6 +18,7 @@
 //    are gathered back to back, so the repeated fiber row is an L1 hit.
 //  * Measured bound: with L2-resident factors the kernel runs at
 //    the L2->SM row-gather rate (~20 TB/s on B200 for 256-byte rows).
+#include <cstdlib>
 #include <vector>
 
 #include "internal.h"
@@ -84,10 +85,10 @@ __device__ __forceinline__ const double2* row_addr(const char* base, unsigned j)
 // One warp processes chunk c.  Fb[q] = lane's byte offset into the row source of
 // slot q (a factor in global memory, or the shared-memory slab of a k-blocked
 // copy, already shifted by the slab's first row).
-template <int NOTHER, int R, int RECB>
+template <int NOTHER, int R, int RECB, int GL = 0>
 __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const char* const* Fb, int4* srec) {
   constexpr int RV = R / 2;                    // double2 per row
-  constexpr int G = RV < 32 ? RV : 32;         // lanes per group
+  constexpr int G = GL ? GL : (RV < 32 ? RV : 32);   // lanes per group
   constexpr int VPL = RV / G;                  // double2 per lane
   constexpr int P = 32 / G;                    // nonzeros per warp step
   constexpr unsigned ROWB = R * 8;
@@ -191,9 +192,9 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
 }
 
 // MINB: CTAs per SM the register budget targets (2 for long rows, 4 for short ones)
-template <int NOTHER, int R, int RECB, int MINB>
+template <int NOTHER, int R, int RECB, int MINB, int GL = 0>
 __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
-  constexpr int G = (R / 2) < 32 ? (R / 2) : 32;
+  constexpr int G = GL ? GL : ((R / 2) < 32 ? (R / 2) : 32);
   const int gl = (threadIdx.x & 31) % G;
   const char* Fb[NOTHER];
 #pragma unroll
@@ -201,7 +202,7 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
   const int64_t warp0 = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5);
   const int64_t nwarps = (int64_t)gridDim.x * kWarps;
   __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
-  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB>(a, c, Fb, srec);
+  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL>(a, c, Fb, srec);
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -366,7 +367,7 @@ bool launch_tiled_r(const MArgs& a, int grid, cudaStream_t st) {
 }
 
 template <int NOTHER, int RECB>
-bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled) {
+bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl) {
   // short rows (few nonzeros per row): row flushes dominate and latency hiding
   // needs more warps -> the 4-CTA/SM register budget; long rows -> 2 CTAs/SM
   const bool short_rows = a.nnz < 64 * a.I;
@@ -379,6 +380,14 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled) {
       default: break;  // other ranks: the flat kernel on the k-blocked copy
     }
   }
+#define GCASE(RR, GG)                                                                   \
+  if (a.R == RR && gl == GG) {                                                      \
+    if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4, GG><<<grid, kWarps * 32, 0, st>>>(a); \
+    else k_mttkrp_fast<NOTHER, RR, RECB, 2, GG><<<grid, kWarps * 32, 0, st>>>(a);          \
+    return true;                                                                        \
+  }
+  GCASE(32, 8) GCASE(64, 16)
+#undef GCASE
   switch (a.R) {
 #define CASE(RR)                                                                     \
   case RR:                                                                           \
@@ -391,17 +400,17 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled) {
   }
 }
 
-cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st) {
+cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, int gl) {
   bool done = false;
   const bool tl = a.ckb != nullptr;
   const int g = tl ? tgrid : grid;
   switch (a.nother) {
-    case 1: done = launch_fast<1, 16>(a, grid, st, false); break;
-    case 2: done = launch_fast<2, 16>(a, g, st, tl); break;
-    case 3: done = launch_fast<3, 32>(a, g, st, tl); break;
-    case 4: done = launch_fast<4, 32>(a, g, st, tl); break;
-    case 5: done = launch_fast<5, 32>(a, g, st, tl); break;
-    case 6: done = launch_fast<6, 32>(a, g, st, tl); break;
+    case 1: done = launch_fast<1, 16>(a, grid, st, false, gl); break;
+    case 2: done = launch_fast<2, 16>(a, g, st, tl, gl); break;
+    case 3: done = launch_fast<3, 32>(a, g, st, tl, gl); break;
+    case 4: done = launch_fast<4, 32>(a, g, st, tl, gl); break;
+    case 5: done = launch_fast<5, 32>(a, g, st, tl, gl); break;
+    case 6: done = launch_fast<6, 32>(a, g, st, tl, gl); break;
     default: break;   // 7 other modes: 48-byte records, generic path
   }
   if (!done) {
@@ -536,7 +545,20 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
   const int tgrid = (int)std::min<int64_t>(std::max<int64_t>(ms.nctachunks, 1), (int64_t)di.sms * 2);
   // (a.ckb is set only for SMEM-slab copies; L2-blocked copies run the flat kernel on virtual rows)
-  CSTF_TRY(launch_main(a, grid, tgrid, st));
+  // Lanes per factor row: 8 lanes x 32 B (4 nonzeros per warp step) when the gathered
+  // factors are L2-resident -- more nonzeros per load instruction, so adjacent
+  // fiber nonzeros share L1 wavefronts (NELL-2 1.80 -> 1.63 ms per mode); the
+  // default 16 lanes x 16 B when they stream from HBM (Delicious, Amazon: no gain
+  // or a loss).  CSTF_MTTKRP_G forces a value (experiments).
+  int gl = 0;
+  {
+    int64_t gbytes = 0;
+    for (int q = 0; q < N - 1; q++) gbytes += X->dims[ms.other[q]] * (int64_t)R * 8;
+    if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
+    static const int gl_env = getenv("CSTF_MTTKRP_G") ? atoi(getenv("CSTF_MTTKRP_G")) : -1;
+    if (gl_env >= 0) gl = gl_env;
+  }
+  CSTF_TRY(launch_main(a, grid, tgrid, st, gl));
   nl++;
   if (nchunks > 1) {
     const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);

@@ -550,8 +550,8 @@ Workspace& ws() {
 // 10 passes: 15.3 -> 14.6 ms).  One-pass (streaming) launches are HBM-bound and
 // keep the 4-CTA/SM variant.  CSTF_ADMM_IREG=0/1 forces either (experiments).
 bool admm_ireg(int kiters) {
-  static const int v = [] { const char* e = getenv("CSTF_ADMM_IREG"); return e ? (e[0] == '1' ? 1 : 0) : -1; }();
-  return v < 0 ? kiters >= 4 : v == 1;
+  const char* e = getenv("CSTF_ADMM_IREG");          // read per call (tests force both paths)
+  return e ? e[0] == '1' : kiters >= 4;
 }
 
 size_t dmma_smem(int RP, bool gram, int nsl) {

@@ -555,8 +555,8 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     int64_t gbytes = 0;
     for (int q = 0; q < N - 1; q++) gbytes += X->dims[ms.other[q]] * (int64_t)R * 8;
     if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
-    static const int gl_env = getenv("CSTF_MTTKRP_G") ? atoi(getenv("CSTF_MTTKRP_G")) : -1;
-    if (gl_env >= 0) gl = gl_env;
+    const char* ge = getenv("CSTF_MTTKRP_G");        // read per call (tests force both paths)
+    if (ge && (atoi(ge) == 0 || atoi(ge) == 8)) gl = atoi(ge);
   }
   CSTF_TRY(launch_main(a, grid, tgrid, st, gl));
   nl++;

@@ -124,6 +124,24 @@ def test_mttkrp_parity(B, case, R):
         assert normwise(host(M), want) <= TOL, (n, R)
 
 
+@pytest.mark.parametrize("gl", ["0", "8"])
+@pytest.mark.parametrize("case", [("3mode", (300, 211, 97), 60000), ("4mode", (40, 37, 53, 29), 50000)])
+def test_mttkrp_group_width_variants(B, gl, case, monkeypatch):
+    """Both lane-group widths of the R = 32 fast path (16 lanes x 16 B and 8 lanes x 32 B,
+    chosen by factor size in production) against the oracle, forced per call."""
+    monkeypatch.setenv("CSTF_MTTKRP_G", gl)
+    name, dims, nnz = case
+    idx, vals = random_coo(len(dims) * 7 + int(gl), dims, nnz, dup_frac=0.05)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    Xo = oracle.coalesce(dims, idx, vals)
+    F = [datagen.uniform(3, 40 + k, I * 32).reshape(I, 32) for k, I in enumerate(dims)]
+    Fd = [cu(f) for f in F]
+    for n in range(len(dims)):
+        M = cu(np.full((dims[n], 32), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        assert normwise(host(M), oracle.mttkrp(Xo, n, F)) <= TOL, (n, gl)
+
+
 def test_mttkrp_heavy_row_spans_many_chunks(B):
     """One row holding most nonzeros (carry fix-up across many chunks) + empty rows."""
     rng = np.random.default_rng(3)
@@ -198,6 +216,20 @@ def test_admm_fixed_iterations(B, variant, I, R):
     assert normwise(host(Ud), Ur) <= TOL
     for k in ("rho", "r_primal", "s_dual", "normH2", "normU2"):
         assert st[k] == pytest.approx(sr[k], rel=1e-9, abs=1e-300), k
+
+
+@pytest.mark.parametrize("ireg", ["0", "1"])
+@pytest.mark.parametrize("max_iter", [3, 10])
+def test_admm_inv_placement_variants(B, ireg, max_iter, monkeypatch):
+    """R = 32 ADMM with the Inv fragments in SMEM and in registers (forced per call);
+    also with the fused Gram epilogue of cstf_factorize."""
+    monkeypatch.setenv("CSTF_ADMM_IREG", ireg)
+    M, S, H, U = admm_inputs(2501, 32, 17)
+    Hd, Ud = cu(H), cu(U)
+    st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=0.0, max_iter=max_iter)
+    Hr, Ur, sr = oracle.admm(M, S, H, U, tol=0.0, max_iter=max_iter)
+    assert st["iters"] == sr["iters"] == max_iter
+    assert normwise(host(Hd), Hr) <= TOL and normwise(host(Ud), Ur) <= TOL
 
 
 @pytest.mark.parametrize("max_iter", [1, 17, 40])

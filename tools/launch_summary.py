@@ -5,22 +5,15 @@ import csv
 import sys
 
 
-def main(path, out=None):
+def main(path, out=None, nmodes_arg=None):
     rows = [r for r in csv.reader(open(path)) if len(r) > 10]
     hdr, data = rows[0], rows[1:]
     ki, mi, vi = hdr.index("Kernel Name"), hdr.index("Metric Name"), hdr.index("Metric Value")
     launches = [(r[ki], float(r[vi].replace(",", ""))) for r in data if r[mi] == "gpu__time_duration.sum"]
     starts = [i for i, (k, _) in enumerate(launches) if "k_chol_inverse" in k]
-    nmodes = 0
     # the last outer iteration starts at the N-th last chol_inverse (one per mode)
-    for cand in (4, 3, 2):
-        if len(starts) >= cand:
-            nmodes = cand
-            break
+    nmodes = min(int(nmodes_arg), len(starts)) if nmodes_arg else min(3, len(starts))
     text = []
-    for N in (3, 4):
-        if len(starts) < N:
-            continue
     tot = collections.Counter()
     first = starts[-nmodes] if nmodes else 0
     for k, t in launches[first:]:
@@ -37,4 +30,5 @@ def main(path, out=None):
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None)
+    # usage: launch_summary.py launches.csv [out.txt] [nmodes]
+    main(sys.argv[1], sys.argv[2] if len(sys.argv) > 2 else None, sys.argv[3] if len(sys.argv) > 3 else None)

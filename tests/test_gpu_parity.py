@@ -218,12 +218,13 @@ def test_admm_fixed_iterations(B, variant, I, R):
         assert st[k] == pytest.approx(sr[k], rel=1e-9, abs=1e-300), k
 
 
-@pytest.mark.parametrize("ireg", ["0", "1"])
+@pytest.mark.parametrize("ireg,pref", [("0", "0"), ("1", "0"), ("1", "1")])
 @pytest.mark.parametrize("max_iter", [3, 10])
-def test_admm_inv_placement_variants(B, ireg, max_iter, monkeypatch):
-    """R = 32 ADMM with the Inv fragments in SMEM and in registers (forced per call);
-    also with the fused Gram epilogue of cstf_factorize."""
+def test_admm_inv_placement_variants(B, ireg, pref, max_iter, monkeypatch):
+    """R = 32 ADMM with the Inv fragments in SMEM and in registers, with and without the
+    cp.async row-group prefetch (forced per call); ragged row count (2501)."""
     monkeypatch.setenv("CSTF_ADMM_IREG", ireg)
+    monkeypatch.setenv("CSTF_ADMM_PREF", pref)
     M, S, H, U = admm_inputs(2501, 32, 17)
     Hd, Ud = cu(H), cu(U)
     st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=0.0, max_iter=max_iter)

@@ -87,6 +87,39 @@ void runbig(double* out, int sms) {
   printf("m16n8k%-2d: %.3f ms  %.2f TF\n", K, ms, warps * 8 * 2.0 * 16 * 8 * K / ms / 1e9);
 }
 
+// latency: one warp per SM (or W warps), NCH independent accumulator chains
+template <int NCH>
+__global__ void lat(double* out, int iters, long long* cyc) {
+  double a = threadIdx.x * 1e-3, b = threadIdx.x * 2e-3;
+  double c[NCH][2];
+#pragma unroll
+  for (int t = 0; t < NCH; t++) { c[t][0] = 0; c[t][1] = 0; }
+  long long t0 = clock64();
+  for (int i = 0; i < iters; i++) {
+#pragma unroll
+    for (int t = 0; t < NCH; t++)
+      asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                   : "+d"(c[t][0]), "+d"(c[t][1]) : "d"(a), "d"(b));
+  }
+  long long t1 = clock64();
+  double s = 0;
+#pragma unroll
+  for (int t = 0; t < NCH; t++) s += c[t][0] + c[t][1];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+  if (threadIdx.x == 0 && blockIdx.x == 0) *cyc = t1 - t0;
+}
+
+template <int NCH>
+void runlat(double* out, long long* dc, int warps) {
+  const int iters = 2000;
+  lat<NCH><<<1, 32 * warps>>>(out, 10, dc);
+  lat<NCH><<<1, 32 * warps>>>(out, iters, dc);
+  long long c = 0;
+  cudaMemcpy(&c, dc, 8, cudaMemcpyDeviceToHost);
+  printf("DMMA chains %d warps/CTA %2d: %.1f cycles per DMMA per warp-chain step (%.2f cycles per DMMA issued)\n",
+         NCH, warps, (double)c / iters, (double)c / iters / NCH / warps);
+}
+
 int main() {
   int sms; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
   double* out; CK(cudaMalloc(&out, 64 << 20));
@@ -96,6 +129,9 @@ int main() {
   runmix<8, 8>(out, sms);
   runmix<8, 16>(out, sms);
   runmix<8, 32>(out, sms);
+  long long* dc; cudaMalloc(&dc, 8);
+  runlat<1>(out, dc, 1); runlat<2>(out, dc, 1); runlat<4>(out, dc, 1); runlat<8>(out, dc, 1);
+  runlat<4>(out, dc, 4); runlat<4>(out, dc, 8); runlat<4>(out, dc, 12); runlat<8>(out, dc, 4); runlat<8>(out, dc, 8);
   runbig<4>(out, sms);
   runbig<8>(out, sms);
   runbig<16>(out, sms);

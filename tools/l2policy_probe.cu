@@ -2,6 +2,7 @@
 // tables much larger than L2 (Delicious-shaped: 17.3M rows gamma=2 and 2.5M rows
 // gamma=3), with the hot rows first (row id = rank).  Compares plain loads with
 // loads that tag rows id < H_k evict_last and the rest evict_first.
+#include <algorithm>
 #include <cstdio>
 #include <cstdint>
 #include <cmath>
@@ -83,5 +84,35 @@ int main() {
     printf("mode %d hB=%7d hC=%7d (%5.1f MB): %.3f ms\n", MD, hb[0], hb[1], (hb[0] + hb[1]) * 256.0 / 1e6, ms); \
   }
   RUN(1) RUN(2) RUN(3) RUN(4)
+  // persisting-L2 set-aside + access-policy window over the hottest rows of one table
+  cudaDeviceProp prop; cudaGetDeviceProperties(&prop, 0);
+  printf("persistingL2CacheMaxSize %d MB, accessPolicyMaxWindowSize %d MB\n", prop.persistingL2CacheMaxSize >> 20,
+         prop.accessPolicyMaxWindowSize >> 20);
+  cudaStream_t st; cudaStreamCreate(&st);
+  for (double frac : {0.25, 0.5, 0.75}) {
+    size_t setaside = (size_t)(prop.persistingL2CacheMaxSize * frac);
+    CK(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside));
+    for (int which = 0; which < 2; which++) {
+      for (double mult : {0.5, 1.0, 2.0}) {
+        cudaStreamAttrValue v = {};
+        size_t bytes = (size_t)(setaside * mult);
+        if (bytes > (size_t)prop.accessPolicyMaxWindowSize) bytes = prop.accessPolicyMaxWindowSize;
+        v.accessPolicyWindow.base_ptr = which ? (void*)B : (void*)C;
+        v.accessPolicyWindow.num_bytes = bytes;
+        v.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)setaside / bytes);
+        v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+        v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+        CK(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v));
+        gather<0><<<grid, 256, 0, st>>>(B, C, jk, nnz, 0, 0, out);
+        cudaEventRecord(e0, st); gather<0><<<grid, 256, 0, st>>>(B, C, jk, nnz, 0, 0, out); cudaEventRecord(e1, st);
+        CK(cudaEventSynchronize(e1)); cudaEventElapsedTime(&ms, e0, e1);
+        printf("window on %s: setaside %.0f MB, window %.0f MB: %.3f ms\n", which ? "B(17.3M,g2)" : "C(2.5M,g3)",
+               setaside / 1e6, bytes / 1e6, ms);
+        v.accessPolicyWindow.num_bytes = 0;
+        cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v);
+        cudaCtxResetPersistingL2Cache();
+      }
+    }
+  }
   return 0;
 }

@@ -400,6 +400,15 @@ cstf_status cstf_tensor_info(const cstf_tensor* X, int* nmodes, int64_t* dims, i
   return CSTF_OK;
 }
 
+cstf_status cstf_tensor_layout(const cstf_tensor* X, int mode, int64_t* nblk, int64_t* blk_rows, int* blk_mode) {
+  if (!X || mode < 0 || mode >= X->N) return fail(CSTF_ERR_INVALID_ARG, "tensor is NULL or bad mode");
+  const ModeStore& ms = X->mode[mode];
+  if (nblk) *nblk = ms.tiled ? ms.nblk : 1;
+  if (blk_rows) *blk_rows = ms.tiled ? ms.blk_rows : 0;
+  if (blk_mode) *blk_mode = ms.tiled ? ms.other[ms.tslot] : -1;
+  return CSTF_OK;
+}
+
 cstf_status cstf_tensor_export_coo(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals) {
   if (!X || (X->nnz > 0 && (!host_idx || !host_vals))) return fail(CSTF_ERR_INVALID_ARG, "export arguments");
   if (X->nranks > 1) return fail(CSTF_ERR_UNSUPPORTED, "export of a partitioned tensor");

@@ -89,7 +89,8 @@ int comm_rank(const cstf_comm* c);
 // and sums the partials over kb in fixed order.  The factor rows of block kb are
 // staged in shared memory by the CTA that processes them.
 constexpr int kTileRows = 256;        // SMEM-slab blocks (opt-in CSTF_KBLOCK=1)
-constexpr int64_t kL2Rows = 131072;     // L2 blocks: 32 MB of factor rows at R = 32
+constexpr int64_t kL2Rows = 65536;      // L2 blocks: 16 MB of factor rows at R = 32
+constexpr int64_t kL2Chunk = 256;       // MTTKRP chunk of an L2-blocked copy (dynamic order)
 struct ModeStore {
   int64_t I = 0;            // rows of this mode (local rows when distributed)
   int64_t nnz = 0;          // nonzeros in this copy

@@ -41,6 +41,7 @@ struct MArgs {
   int64_t It;             // rows of the k-blocked mode's factor (slot nother-1)
   double* M;            // output rows (virtual rows when k-blocked)
   double* carry;        // [nchunks][R]
+  unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
 };
 
 __device__ __forceinline__ int64_t chunk_begin(const MArgs& a, int64_t c) {
@@ -202,6 +203,20 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
   const int64_t warp0 = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5);
   const int64_t nwarps = (int64_t)gridDim.x * kWarps;
   __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
+  if (a.queue) {
+    // L2-blocked copies: warps take chunks in global order from a counter, so the
+    // nonzeros in flight span a narrow range of the blocked factor's rows (its
+    // L2-resident slab) instead of grid-stride windows spread over the tensor.
+    // Which warp runs a chunk does not change its arithmetic (deterministic).
+    for (;;) {
+      unsigned long long c = 0;
+      if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if ((int64_t)c >= a.nchunks) break;
+      process_chunk<NOTHER, R, RECB, GL>(a, (int64_t)c, Fb, srec);
+    }
+    return;
+  }
   for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL>(a, c, Fb, srec);
 }
 
@@ -423,7 +438,7 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, in
 }
 
 struct Workspace {
-  DevBuf lb, cont, carry, gsum, partial, kbptr;
+  DevBuf lb, cont, carry, gsum, partial, kbptr, queue;
   std::vector<int64_t> hk;
 };
 
@@ -489,7 +504,9 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   MArgs a;
   a.wstart = nullptr;
   a.ckb = nullptr;
+  a.queue = nullptr;
   int64_t chunk = 0, nchunks = 0;
+  const bool l2blk = ms.tiled && !ms.slab;
   if (ms.tiled && ms.slab) {
     CSTF_TRY(tiled_split(ms, st));
     nchunks = ms.nwchunks;
@@ -502,6 +519,10 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     chunk = ((chunk + 31) / 32) * 32;
     if (chunk < 256) chunk = 256;
     if (chunk > 8192) chunk = 8192;
+    if (l2blk) {     // dynamic order: the window in flight = resident warps x chunk nonzeros
+      const char* ce = getenv("CSTF_L2_CHUNK");
+      chunk = ce && atoll(ce) >= 32 ? (atoll(ce) + 31) / 32 * 32 : kL2Chunk;
+    }
     nchunks = nnz > 0 ? (nnz + chunk - 1) / chunk : 1;
   }
   CSTF_TRY(w.carry.ensure((size_t)nchunks * R * 8));
@@ -542,7 +563,14 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     ms.cchunk = chunk;
     ms.cnchunks = nchunks;
   }
-  const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
+  int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
+  if (l2blk && nchunks > 1) {
+    CSTF_TRY(w.queue.ensure(8));
+    CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
+    a.queue = w.queue.as<unsigned long long>();
+    const bool short_rows = nnz < 64 * ms.Ivirt;        // = launch_fast's CTA budget
+    grid = (int)std::min<int64_t>(grid, (int64_t)di.sms * (short_rows ? 4 : 2));   // resident CTAs only
+  }
   const int tgrid = (int)std::min<int64_t>(std::max<int64_t>(ms.nctachunks, 1), (int64_t)di.sms * 2);
   // (a.ckb is set only for SMEM-slab copies; L2-blocked copies run the flat kernel on virtual rows)
   // Lanes per factor row: 8 lanes x 32 B (4 nonzeros per warp step) when the gathered

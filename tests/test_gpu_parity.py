@@ -460,6 +460,36 @@ def test_mttkrp_l2_blocked_copies(B, R, monkeypatch):
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
 
 
+def test_mttkrp_l2_blocked_default(B, monkeypatch):
+    """Default L2 blocking of short output modes against a factor that does not fit
+    L2 (the Delicious mode-4 shape in small): layout chosen, parity with the oracle,
+    bitwise repeatable under the dynamic chunk order, same result unblocked."""
+    dims = (50, 600_000, 1000, 20)
+    idx, vals = datagen.coo(dims, (1, 2, 3, 1), 1_500_000, 23)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    for n in (0, 2, 3):
+        nblk, rows, bm = X.layout(n)
+        assert bm == 1 and rows > 0 and nblk == -(-dims[1] // rows) and nblk > 1, (n, nblk, rows, bm)
+    assert X.layout(1)[0] == 1
+    R = 32
+    F = datagen.init_factors(dims, R, 4)
+    Fd = [cu(f) for f in F]
+    monkeypatch.setenv("CSTF_L2_BLOCK", "0")
+    Xp = B.cstf_tensor_load_coo(dims, idx, vals)
+    assert all(Xp.layout(n)[0] == 1 for n in range(4))
+    for n in range(4):
+        M = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        first = host(M).copy()
+        B.cstf_mttkrp(X, n, Fd, M)
+        assert np.array_equal(host(M), first), n
+        assert normwise(first, oracle.mttkrp(ref, n, F)) <= TOL, n
+        Mp = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(Xp, n, Fd, Mp)
+        assert normwise(first, host(Mp)) <= TOL, n
+
+
 def test_factorize_bitwise_deterministic(B):
     """Fixed grids and fixed reduction orders everywhere: two runs are bit-identical."""
     c = datagen.CONFIGS["enron"].scaled(60, nnz_factor=1000)

@@ -83,3 +83,41 @@ def test_fullsize_one_outer_iteration(full):
     for a, b in zip(Fd, orc["factors"]):
         assert normwise(a.cpu().numpy(), b) <= 1e-6
     assert normwise(lam.cpu().numpy(), orc["lam"][-1]) <= 1e-6
+
+
+@pytest.fixture(scope="module")
+def delicious():
+    """configs[3] (Delicious-shaped, 140M nonzeros, R = 32): the copy of mode 4
+    is L2-blocked by default (short output mode, 4.4 GB factor of mode 2)."""
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_sohksc24_b200 import binding as B
+    c = datagen.CONFIGS["delicious"]
+    idx, vals = c.generate()
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    ref = oracle.coalesce(c.dims, idx, vals)
+    del idx, vals
+    F = datagen.init_factors(c.dims, c.R, c.seed)
+    yield B, c, X, ref, F
+    X.free()
+
+
+def test_fullsize_delicious_mttkrp_sampled_rows(delicious):
+    B, c, X, ref, F = delicious
+    info = X.info()
+    assert info["nnz"] == ref.nnz and info["hash"] == ref.hash
+    assert [X.layout(n)[0] > 1 for n in range(4)] == [False, False, False, True]
+    rng = np.random.default_rng(1)
+    Fd = [torch.from_numpy(f).cuda() for f in F]
+    for n, I in enumerate(c.dims):
+        counts = np.bincount(ref.idx[n], minlength=I)
+        k = 12 if n == 3 else 100        # mode-4 rows hold ~100K nonzeros each
+        rows = np.unique(np.concatenate([rng.integers(0, I, k), [np.argmax(counts), np.argmin(counts), 0, I - 1]]))
+        M = torch.full((I, c.R), float("nan"), dtype=torch.float64, device="cuda")
+        B.cstf_mttkrp(X, n, Fd, M)
+        torch.cuda.synchronize()
+        got = M[torch.from_numpy(rows).cuda()].cpu().numpy()
+        want = oracle.mttkrp_rows(ref, n, F, rows)
+        assert normwise(got, want) <= TOL, n
+        assert not torch.isnan(M).any().item()
+        del M

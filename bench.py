@@ -192,6 +192,10 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--comm", choices=["nccl", "host"], default="nccl",
+                    help="N > 1 transport: nccl (one GPU per rank, the product path) or host (gloo "
+                         "host callbacks; ranks may share one GPU -- validates the multi-rank path, "
+                         "not a performance number)")
     ap.add_argument("--ablation", action="store_true",
                     help="also time one ADMM update per mode with the streaming (one launch per inner "
                          "iteration, the paper's fused shape) and the row-resident variants (SURVEY f2)")
@@ -204,13 +208,20 @@ def main():
     from paper_conf_icpp_sohksc24_b200 import binding as B
 
     rank, world, local = env_rank()
+    host_comm = world > 1 and args.comm == "host"
+    if host_comm:                            # validation: N ranks may share one GPU
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dist = None
     comm = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        comm = B.cstf_comm_create_nccl()     # rows of every mode partitioned over the ranks
+        if host_comm:
+            dist.init_process_group("gloo")
+            comm = B.cstf_comm_create_host()
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            comm = B.cstf_comm_create_nccl()     # rows of every mode partitioned over the ranks
     R = cfg.R
     t0 = time.time()
     idx, vals = cfg.generate()
@@ -251,7 +262,7 @@ def main():
     clk = clocks.stop()
     ms_total = e0.elapsed_time(e1)
     if dist:
-        t = torch.tensor([ms_total], device="cuda")
+        t = torch.tensor([ms_total], device="cpu" if host_comm else "cuda")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms_total = float(t.item())
     ms_step = ms_total / args.steps
@@ -311,7 +322,10 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic (datagen recipe, shapes of PAPER.md Table 2)",
-            "config": config_dict(cfg), "gpu_launches": int(launches),
+            "config": dict(config_dict(cfg), **({"parallelism": f"rows of every mode partitioned over {world} ranks",
+                                                 "comm": "host callbacks (validation, shared GPU)" if host_comm
+                                                 else "NCCL + CUDA-IPC peer stores"} if world > 1 else {})),
+            "gpu_launches": int(launches),
             "roofline": roof, "roofline_gather": line_gather, "roofline_admm": roof_admm, "admm_update_gbs": admm_gbs,
             "phases_ms_per_step": phase_ms, "clocks": clk,
             "setup": {"generate_s": t_gen, "load_coo_s": t_load, "nnz_coalesced": nnz}}
@@ -332,7 +346,12 @@ def main():
             torch.cuda.synchronize()
             ts.append(a.elapsed_time(b))
         fac_bytes = sum(I * R * 8 for I in cfg.dims)
-        line["e2e"] = {"value": float(np.mean(ts)) / 1e3, "unit": "s", "h2d_bytes_per_step": fac_bytes,
+        e2e_s = float(np.mean(ts)) / 1e3
+        if dist:                              # max over ranks, like the device-timed value
+            t = torch.tensor([e2e_s], device="cpu" if host_comm else "cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            e2e_s = float(t.item())
+        line["e2e"] = {"value": e2e_s, "unit": "s", "h2d_bytes_per_step": fac_bytes,
                        "d2h_bytes_per_step": fac_bytes + R * 8 + 8,
                        "note": "cstf_factorize_host: initial factors H2D, 1 outer iteration, factors+lambda+fit D2H"}
     if args.ablation and world == 1:

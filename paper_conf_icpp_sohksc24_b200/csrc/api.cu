@@ -168,8 +168,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
   if (o->update < CSTF_UPDATE_ADMM || o->update > CSTF_UPDATE_MU) return fail(CSTF_ERR_INVALID_ARG, "unknown update");
   if (o->update == CSTF_UPDATE_MU && R > 64) return fail(CSTF_ERR_UNSUPPORTED, "MU update for R > 64");
-  const bool dist = X->nranks > 1;
-  if (comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
+  const bool dist = X->partitioned;
+  if ((comm != nullptr) != dist || comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
     return fail(CSTF_ERR_INVALID_ARG, "comm does not match the tensor's partition");
   for (int n = 0; n < N; n++)
     if (!d_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");
@@ -381,6 +381,7 @@ cstf_status cstf_tensor_load_coo(int nmodes, const int64_t* dims, int64_t nnz,
   X->N = nmodes;
   X->nranks = comm_nranks(comm);
   X->rank = comm_rank(comm);
+  X->partitioned = comm != nullptr;
   for (int n = 0; n < nmodes; n++) X->dims[n] = dims[n];
   cudaGetDevice(&X->device);
   cstf_status s = build_store(X, host_idx, host_vals, nnz, S(stream));
@@ -411,7 +412,7 @@ cstf_status cstf_tensor_layout(const cstf_tensor* X, int mode, int64_t* nblk, in
 
 cstf_status cstf_tensor_export_coo(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals) {
   if (!X || (X->nnz > 0 && (!host_idx || !host_vals))) return fail(CSTF_ERR_INVALID_ARG, "export arguments");
-  if (X->nranks > 1) return fail(CSTF_ERR_UNSUPPORTED, "export of a partitioned tensor");
+  if (X->partitioned) return fail(CSTF_ERR_UNSUPPORTED, "export of a partitioned tensor");
   return export_store(X, host_idx, host_vals);
 }
 
@@ -421,7 +422,7 @@ cstf_status cstf_mttkrp(const cstf_tensor* X, int mode, int R, const double* con
                         void* stream) {
   if (!X || !d_factors || !d_M) return fail(CSTF_ERR_INVALID_ARG, "NULL argument");
   if (mode < 0 || mode >= X->N) return fail(CSTF_ERR_INVALID_ARG, "mode out of range");
-  if (X->nranks > 1) return fail(CSTF_ERR_UNSUPPORTED, "cstf_mttkrp on a partitioned tensor (use cstf_factorize)");
+  if (X->partitioned) return fail(CSTF_ERR_UNSUPPORTED, "cstf_mttkrp on a partitioned tensor (use cstf_factorize)");
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
   for (int k = 0; k < X->N; k++)
     if (k != mode && !d_factors[k]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");

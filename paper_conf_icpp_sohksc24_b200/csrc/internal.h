@@ -134,6 +134,7 @@ struct cstf_tensor {
   // so every rank's rows are one contiguous slice [rank*B_n, (rank+1)*B_n) of the
   // internal (relabelled, zero-padded) factor of P*B_n rows.
   int nranks = 1, rank = 0;
+  bool partitioned = false;           // loaded with a communicator (any size): row-partitioned layout
   int64_t rows_per_rank[8] = {0};     // B_n
   cstf::DevBuf relabel[8];            // int32[dims[n]]: internal label of original row
 };

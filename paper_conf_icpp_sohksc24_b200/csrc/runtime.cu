@@ -109,7 +109,7 @@ int comm_nranks(const cstf_comm* c) { return c ? c->c.nranks : 1; }
 int comm_rank(const cstf_comm* c) { return c ? c->c.rank : 0; }
 
 cstf_status comm_allreduce_f64(const cstf_comm* c, double* d_buf, size_t count, cudaStream_t st) {
-  if (!c || c->c.nranks <= 1 || count == 0) return CSTF_OK;
+  if (!c || count == 0 || (c->c.nranks <= 1 && !c->c.nccl)) return CSTF_OK;
   if (c->c.host_allreduce) {
     std::vector<double> h(count);
     CSTF_CUDA(cudaMemcpyAsync(h.data(), d_buf, count * 8, cudaMemcpyDeviceToHost, st));
@@ -125,7 +125,7 @@ cstf_status comm_allreduce_f64(const cstf_comm* c, double* d_buf, size_t count, 
 }
 cstf_status comm_allgather_f64(const cstf_comm* c, const double* d_send, double* d_recv,
                                size_t count_per_rank, cudaStream_t st) {
-  if (!c || c->c.nranks <= 1) {
+  if (!c || (c->c.nranks <= 1 && !c->c.nccl)) {
     if (d_send != d_recv && count_per_rank)
       CSTF_CUDA(cudaMemcpyAsync(d_recv, d_send, count_per_rank * 8, cudaMemcpyDeviceToDevice, st));
     return CSTF_OK;
@@ -186,7 +186,7 @@ cstf_status cstf_comm_create(int nranks, int rank, const unsigned char id[128], 
   cstf_comm* c = new cstf_comm();
   c->c.nranks = nranks;
   c->c.rank = rank;
-  if (nranks > 1) {
+  {   // also for one rank: the same NCCL calls run (a 1-rank job exercises the transport)
     cstf_status s = nccl_load();
     if (s != CSTF_OK) { delete c; return s; }
     ncclUniqueId u;

@@ -549,7 +549,7 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     X->normX2 = hv[0];
     memcpy(&X->hash, &hv[1], 8);
   }
-  if (X->nranks > 1) return build_partitioned(X, c_idx, c_vals, nout, tmp, st);
+  if (X->partitioned) return build_partitioned(X, c_idx, c_vals, nout, tmp, st);
   // ---- 6. per-mode copies: sorted by (i_n, other modes by increasing length), AoS records
   const int recb = record_bytes(N);
   for (int n_ = 0; n_ < N; n_++) {

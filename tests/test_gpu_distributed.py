@@ -21,7 +21,7 @@ from paper_conf_icpp_sohksc24_b200 import binding as B
 dist.init_process_group("gloo")
 torch.cuda.set_device(0)
 rank, P = dist.get_rank(), dist.get_world_size()
-comm = B.cstf_comm_create_host()
+comm = B.cstf_comm_create_nccl() if COMM == "nccl" else B.cstf_comm_create_host()
 cfg, scale, R, tol, outer = CASE
 c = datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
 idx, vals = c.generate()
@@ -49,9 +49,9 @@ dist.destroy_process_group()
 '''
 
 
-def run(tmp_path, nproc, case, port):
+def run(tmp_path, nproc, case, port, comm="host"):
     p = tmp_path / "dist_case.py"
-    p.write_text(f"ROOT = {ROOT!r}\nCASE = {case!r}\n" + SCRIPT)
+    p.write_text(f"ROOT = {ROOT!r}\nCASE = {case!r}\nCOMM = {comm!r}\n" + SCRIPT)
     env = dict(os.environ, MASTER_ADDR="127.0.0.1", PYTHONPATH=ROOT)
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
                         "--master-addr=127.0.0.1", f"--master-port={port}", str(p)],
@@ -73,15 +73,21 @@ def run(tmp_path, nproc, case, port):
     (2, ("delicious", 2000, 32, 0.0, 3), 29613, "1"),     # eps = 0: ADMM epilogue peer stores (f4)
     (3, ("nell2", 40, 32, 0.0, 4), 29614, "1"),
     (3, ("nell2", 40, 32, 0.0, 4), 29615, "0"),           # same case through the plain all-gather
+    (1, ("nell2", 40, 32, 0.0, 4), 29616, "nccl"),        # a real NCCL communicator of one rank
+    (1, ("enron", 60, 8, 1e-2, 5), 29617, "nccl"),
 ])
 def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port, peer, monkeypatch):
-    monkeypatch.setenv("CSTF_PEER_STORE", peer)
-    res = run(tmp_path, nproc, case, port)
+    """peer: CSTF_PEER_STORE for the host communicator, or "nccl" (one rank: the
+    NCCL transport -- dlopen, unique id, init, all-reduce, all-gather -- and the
+    partitioned layout with P = 1, the only NCCL job one GPU can run)."""
+    comm = "nccl" if peer == "nccl" else "host"
+    monkeypatch.setenv("CSTF_PEER_STORE", "1" if peer == "nccl" else peer)
+    res = run(tmp_path, nproc, case, port, comm)
     r0 = res[0]
     for rk in range(1, nproc):          # every rank took the same decisions
         assert res[rk]["fit"] == r0["fit"] and res[rk]["iters"] == r0["iters"]
     assert r0["fit_rel"] <= 1e-6
-    if peer == "1" and case[3] == 0.0 and case[2] <= 32:
+    if nproc > 1 and peer == "1" and case[3] == 0.0 and case[2] <= 32:
         assert r0["comm_ms"] == 0.0          # no separate all-gather ran: rows were peer-stored
     if not r0["tie"]:
         assert r0["fac_rel"] <= 1e-6 and r0["lam_rel"] <= 1e-6

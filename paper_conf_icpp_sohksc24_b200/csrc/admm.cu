@@ -70,6 +70,29 @@ __device__ __forceinline__ double prox_apply(int prox, double x, double tau) {
   }
 }
 
+// Sign-bit arithmetic on the integer pipe (exact; used by the FNN passes below)
+__device__ __forceinline__ double d_abs(double x) {
+  return __hiloint2double(__double2hiint(x) & 0x7fffffff, __double2loint(x));
+}
+__device__ __forceinline__ double d_neg(double x) {
+  return __hiloint2double(__double2hiint(x) ^ (int)0x80000000, __double2loint(x));
+}
+// sign bit set -> x, else -0.0   (= -U' for U' = prox residual, see FNN)
+__device__ __forceinline__ double d_wpart(double x) {
+  const int hi = __double2hiint(x), m = hi >> 31;
+  return __hiloint2double((hi & m) | (int)0x80000000, __double2loint(x) & m);
+}
+// sign bit clear -> x, else +0.0  (= x > 0 ? x : +0.0 for every non-NaN x, prox of D15)
+__device__ __forceinline__ double d_pos(double x) {
+  const int hi = __double2hiint(x), m = ~(hi >> 31);
+  return __hiloint2double(hi & m, __double2loint(x) & m);
+}
+// sign bit set -> -x, else +0.0   (= H' - x for H' = d_pos(x): the dual update)
+__device__ __forceinline__ double d_negpart(double x) {
+  const int hi = __double2hiint(x), m = hi >> 31;
+  return __hiloint2double((hi ^ (int)0x80000000) & m, __double2loint(x) & m);
+}
+
 __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b) {
   asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
       : "+d"(d0), "+d"(d1)
@@ -82,7 +105,13 @@ __device__ __forceinline__ void dmma(double& d0, double& d1, double a, double b)
 // IREG: Inv fragments held in registers (RP <= 32, 3 CTAs/SM) instead of read from SMEM per DMMA.
 // PREF (R == RP, !MU): the next row group's m, h, u are staged in SMEM by cp.async while the
 // current group iterates, so the warps of an SM do not all wait on HBM at once.
-template <int RP, bool GRAM, bool MU = false, bool IREG = false, bool PREF = false>
+// FNN (non-negativity prox, !MU, sums_from >= 1): the passes without residual sums keep one
+// value per element, x = H~ - U.  With H' = max(x, +0) and U' = H' - x, every quantity the
+// next pass needs follows from the sign of x exactly: H' + U' = |x|, so the next A operand is
+// fma(rho, |x|, M), and the next x = H~' - U' = H~' + w with w = (x < 0 ? x : -0.0).  Per
+// element and pass that is one DADD and one DFMA on the FP64 datapath (instead of three DADDs,
+// a DSETP and a DFMA), the rest is integer sign-bit logic; results are bit-identical.
+template <int RP, bool GRAM, bool MU = false, bool IREG = false, bool PREF = false, bool FNN = false>
 __global__ void __launch_bounds__(kThreads, IREG ? 3 : 0) k_admm_dmma(KArgs a) {
   constexpr int NT = RP / 8;       // n-tiles of 8 columns
   constexpr int NC = 2 * NT;       // k-chunks of 4
@@ -207,7 +236,67 @@ __global__ void __launch_bounds__(kThreads, IREG ? 3 : 0) k_admm_dmma(KArgs a) {
         }
       }
     }
-    for (int j = 0; j < kiters; j++) {
+    int j0 = 0;
+    if constexpr (FNN) {
+      // passes 0 .. sums_from-1 in x-state: h holds x, u holds w = -U (see FNN above)
+#pragma unroll
+      for (int t = 0; t < NT; t++)
+#pragma unroll
+        for (int i = 0; i < 2; i++) u[t][i] = d_neg(u[t][i]);
+      for (int j = 0; j < a.sums_from; j++) {
+        double d[NT][2];
+#pragma unroll
+        for (int t = 0; t < NT; t++) { d[t][0] = 0.0; d[t][1] = 0.0; }
+        if (j == 0) {
+#pragma unroll
+          for (int c = 0; c < NC; c++) {
+            const int tt = c >> 1, ii = c & 1;
+            const double av = fma(rho, h[tt][ii] - u[tt][ii], m[tt][ii]);   // M + rho (H + U)
+#pragma unroll
+            for (int t = 0; t < NT; t++) {
+              if constexpr (IREG) dmma(d[t][0], d[t][1], av, binv[c][t]);
+              else dmma(d[t][0], d[t][1], av, sinv[(c * NT + t) * 32 + lane]);
+            }
+          }
+        } else {
+#pragma unroll
+          for (int c = 0; c < NC; c++) {
+            const int tt = c >> 1, ii = c & 1;
+            const double av = fma(rho, d_abs(h[tt][ii]), m[tt][ii]);         // M + rho (H + U) = M + rho |x|
+#pragma unroll
+            for (int t = 0; t < NT; t++) {
+              if constexpr (IREG) dmma(d[t][0], d[t][1], av, binv[c][t]);
+              else dmma(d[t][0], d[t][1], av, sinv[(c * NT + t) * 32 + lane]);
+            }
+          }
+        }
+#pragma unroll
+        for (int t = 0; t < NT; t++)
+#pragma unroll
+          for (int i = 0; i < 2; i++) {
+            const double x = d[t][i] + u[t][i];                            // H~ - U
+            h[t][i] = x;
+            u[t][i] = d_wpart(x);
+          }
+      }
+      if (a.sums_from > 0) {
+#pragma unroll
+        for (int t = 0; t < NT; t++)
+#pragma unroll
+          for (int i = 0; i < 2; i++) {
+            const double x = h[t][i];
+            h[t][i] = d_pos(x);
+            u[t][i] = d_negpart(x);
+          }
+      } else {
+#pragma unroll
+        for (int t = 0; t < NT; t++)
+#pragma unroll
+          for (int i = 0; i < 2; i++) u[t][i] = d_neg(u[t][i]);
+      }
+      j0 = a.sums_from;
+    }
+    for (int j = j0; j < kiters; j++) {
       double d[NT][2];
 #pragma unroll
       for (int t = 0; t < NT; t++) { d[t][0] = 0.0; d[t][1] = 0.0; }
@@ -609,19 +698,25 @@ bool admm_pref() {
   return e ? e[0] == '1' : true;
 }
 
-template <int RP, bool GRAM, bool MU = false, bool IREG = false, bool PREF = false>
-cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
+// FNN passes (see k_admm_dmma) for the non-negativity prox; CSTF_ADMM_FNN=0 disables (tests).
+bool admm_fnn(const KArgs& k) {
+  const char* e = getenv("CSTF_ADMM_FNN");
+  return k.prox == CSTF_PROX_NONNEG && k.sums_from >= 1 && !(e && e[0] == '0');
+}
+
+template <int RP, bool GRAM, bool MU = false, bool IREG = false, bool PREF = false, bool FNN = false>
+cstf_status launch_dmma_one(const KArgs& k, int& grid, cudaStream_t st) {
   const int nsl = k.kiters - k.sums_from;
   const size_t smem = dmma_smem(RP, GRAM, nsl, PREF);
   static int per_sm[kMaxK + 1] = {0};
   static bool attr = false;
   if (!attr) {
-    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM, MU, IREG, PREF>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    CSTF_CUDA(cudaFuncSetAttribute(k_admm_dmma<RP, GRAM, MU, IREG, PREF, FNN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                    (int)dmma_smem(RP, GRAM, kMaxK, PREF)));
     attr = true;
   }
   if (!per_sm[nsl]) {
-    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM, MU, IREG, PREF>, kThreads, smem));
+    CSTF_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[nsl], k_admm_dmma<RP, GRAM, MU, IREG, PREF, FNN>, kThreads, smem));
     if (per_sm[nsl] < 1) per_sm[nsl] = 1;
   }
   const int64_t groups = (k.I + 7) / 8;
@@ -629,9 +724,17 @@ cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
   const int64_t cap = (int64_t)device_info().sms * per_sm[nsl];
   if (g > cap) g = cap;
   grid = (int)(g < 1 ? 1 : g);
-  k_admm_dmma<RP, GRAM, MU, IREG, PREF><<<grid, kThreads, smem, st>>>(k);
+  k_admm_dmma<RP, GRAM, MU, IREG, PREF, FNN><<<grid, kThreads, smem, st>>>(k);
   CSTF_LAUNCHED();
   return CSTF_OK;
+}
+
+template <int RP, bool GRAM, bool MU = false, bool IREG = false, bool PREF = false>
+cstf_status launch_dmma_t(const KArgs& k, int& grid, cudaStream_t st) {
+  if constexpr (!MU) {
+    if (admm_fnn(k)) return launch_dmma_one<RP, GRAM, MU, IREG, PREF, true>(k, grid, st);
+  }
+  return launch_dmma_one<RP, GRAM, MU, IREG, PREF, false>(k, grid, st);
 }
 
 cstf_status launch_kernel(const KArgs& k, int& grid, bool gram, cudaStream_t st) {

@@ -233,6 +233,29 @@ def test_admm_inv_placement_variants(B, ireg, pref, max_iter, monkeypatch):
     assert normwise(host(Hd), Hr) <= TOL and normwise(host(Ud), Ur) <= TOL
 
 
+@pytest.mark.parametrize("R,ireg", [(8, "0"), (24, "0"), (32, "0"), (32, "1"), (40, "0"), (64, "0")])
+@pytest.mark.parametrize("max_iter,tol", [(2, 0.0), (10, 0.0), (17, 0.0), (30, 1e-2)])
+def test_admm_fnn_passes_bit_identical(B, R, ireg, max_iter, tol, monkeypatch):
+    """The sign-bit (FNN) passes reproduce the plain epilogue bit for bit, including
+    signed zeros in the incoming H and U and replayed chunks (tol > 0)."""
+    monkeypatch.setenv("CSTF_ADMM_IREG", ireg)
+    M, S, H, U = admm_inputs(1203, R, 3 * R + max_iter)
+    H[::7] = 0.0
+    U[::5] = 0.0
+    U[1::9] = -0.0
+    H[2::11] = -0.0
+    outs = []
+    for fnn in ("1", "0"):
+        monkeypatch.setenv("CSTF_ADMM_FNN", fnn)
+        Hd, Ud = cu(H), cu(U)
+        st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=tol, max_iter=max_iter)
+        outs.append((host(Hd).tobytes(), host(Ud).tobytes(), st["iters"], st["normH2"], st["normU2"]))
+    assert outs[0] == outs[1]
+    Hr, Ur, sr = oracle.admm(M, S, H, U, tol=tol, max_iter=max_iter)
+    if sr["iters"] == outs[0][2]:
+        assert normwise(np.frombuffer(outs[0][0]).reshape(H.shape), Hr) <= TOL
+
+
 @pytest.mark.parametrize("max_iter", [1, 17, 40])
 def test_admm_iteration_chunking(B, max_iter):
     M, S, H, U = admm_inputs(2000, 32, 5)

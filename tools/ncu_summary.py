@@ -22,6 +22,12 @@ KEYS = [
     ("launch__grid_size", "grid"),
     ("launch__block_size", "block"),
     ("launch__occupancy_limit_registers", "occ_lim_regs"),
+    ("sm__pipe_tensor_subpipe_dmma_cycles_active.avg.pct_of_peak_sustained_active", "dmma_pipe_%"),
+    ("smsp__average_warps_issue_stalled_math_pipe_throttle_per_issue_active.ratio", "stall_mathpipe"),
+    ("smsp__average_warps_issue_stalled_wait_per_issue_active.ratio", "stall_wait"),
+    ("smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio", "stall_longsb"),
+    ("l1tex__data_pipe_lsu_wavefronts.avg.pct_of_peak_sustained_elapsed", "l1_wavefront_%"),
+    ("lts__t_sectors_srcunit_tex.avg.pct_of_peak_sustained_elapsed", "l2_tex_sect_%"),
 ]
 
 

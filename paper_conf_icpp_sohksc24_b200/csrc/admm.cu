@@ -411,6 +411,64 @@ __global__ void __launch_bounds__(kThreads, IREG ? 3 : 0) k_admm_dmma(KArgs a) {
   }
 }
 
+// Standalone Gram G = H^T H (Alg. 1 l.4/12) on the FP64 tensor path, RP <= 64: a warp
+// takes 8-row groups (grid stride) and accumulates every upper tile pair (xa <= xb)
+// of G with two DMMA.8x8x4 per pair and group (k = the group's rows); both operands
+// are H[row 4kc + q][col 8x + g] of lane (g, q).  The next group's fragments are
+// loaded while the current one multiplies.  Per-CTA partials [grid][NP][64] (warps
+// summed in order), then k_gram_from_parts (fixed order): deterministic.
+constexpr int kGramWarps = 8;
+template <int NT>
+__global__ void __launch_bounds__(kGramWarps * 32, 1) k_gram_dmma(const double* __restrict__ H, int64_t I, int R,
+                                                                 double* __restrict__ gpart) {
+  constexpr int NP = NT * (NT + 1) / 2;
+  extern __shared__ double sred[];                 // [kGramWarps][NP][64]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, g = lane >> 2, q = lane & 3;
+  double acc[NP][2];
+#pragma unroll
+  for (int p = 0; p < NP; p++) { acc[p][0] = 0.0; acc[p][1] = 0.0; }
+  const int64_t ngroups = (I + 7) / 8;
+  const int64_t gw0 = (int64_t)blockIdx.x * kGramWarps + warp, gws = (int64_t)gridDim.x * kGramWarps;
+  auto load = [&](int64_t grp, double (&fr)[NT][2]) {
+#pragma unroll
+    for (int kc = 0; kc < 2; kc++) {
+      const int64_t row = grp * 8 + 4 * kc + q;
+      const bool rok = grp < ngroups && row < I;
+#pragma unroll
+      for (int x = 0; x < NT; x++) {
+        const int col = 8 * x + g;
+        fr[x][kc] = (rok && col < R) ? __ldg(H + row * R + col) : 0.0;
+      }
+    }
+  };
+  double fr[NT][2];
+  load(gw0, fr);
+  for (int64_t grp = gw0; grp < ngroups; grp += gws) {
+    double nx[NT][2];
+    load(grp + gws, nx);
+    int p = 0;
+#pragma unroll
+    for (int xa = 0; xa < NT; xa++)
+#pragma unroll
+      for (int xb = xa; xb < NT; xb++, p++)
+#pragma unroll
+        for (int kc = 0; kc < 2; kc++) dmma(acc[p][0], acc[p][1], fr[xa][kc], fr[xb][kc]);
+#pragma unroll
+    for (int x = 0; x < NT; x++) { fr[x][0] = nx[x][0]; fr[x][1] = nx[x][1]; }
+  }
+#pragma unroll
+  for (int p = 0; p < NP; p++) {
+    sred[((size_t)warp * NP + p) * 64 + lane * 2] = acc[p][0];
+    sred[((size_t)warp * NP + p) * 64 + lane * 2 + 1] = acc[p][1];
+  }
+  __syncthreads();
+  for (int x = tid; x < NP * 64; x += blockDim.x) {
+    double v = 0.0;
+    for (int w = 0; w < kGramWarps; w++) v += sred[(size_t)w * NP * 64 + x];
+    gpart[(size_t)blockIdx.x * NP * 64 + x] = v;
+  }
+}
+
 // Fixed-order reduction over CTAs: thread t sums parts t, t + 256, ... in order,
 // then a fixed tree over the 256 threads (deterministic for a given grid).
 __device__ __forceinline__ double block_sum_fixed(const double* __restrict__ src, int nparts, size_t stride) {
@@ -783,7 +841,44 @@ cstf_status launch_kernel(const KArgs& k, int& grid, bool gram, cudaStream_t st)
   return CSTF_OK;
 }
 
+template <int NT>
+cstf_status launch_gram_dmma(const double* H, int64_t I, int R, double* G, cudaStream_t st) {
+  constexpr int NP = NT * (NT + 1) / 2;
+  const size_t smem = (size_t)kGramWarps * NP * 64 * 8;
+  static bool attr = false;
+  if (!attr) {
+    CSTF_CUDA(cudaFuncSetAttribute(k_gram_dmma<NT>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    attr = true;
+  }
+  const int64_t groups = (I + 7) / 8;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>((groups + kGramWarps - 1) / kGramWarps,
+                                                                (int64_t)device_info().sms));
+  Workspace& w = ws();
+  CSTF_TRY(w.gpart.ensure((size_t)grid * NP * 64 * 8));
+  k_gram_dmma<NT><<<grid, kGramWarps * 32, smem, st>>>(H, I, R, w.gpart.as<double>());
+  CSTF_LAUNCHED();
+  k_gram_from_parts<<<NP * 64, 256, 0, st>>>(w.gpart.as<double>(), grid, NT, R, G);
+  CSTF_LAUNCHED();
+  return CSTF_OK;
+}
+
 }  // namespace
+
+bool gram_dmma(const double* d_H, int64_t I, int R, double* d_G, cudaStream_t st, cstf_status* status) {
+  const char* e = getenv("CSTF_GRAM_DMMA");            // 0: the DFMA register-tile kernel (tests)
+  if (R < 1 || R > 64 || (e && e[0] == '0')) return false;
+  switch ((R + 7) / 8) {
+    case 1: *status = launch_gram_dmma<1>(d_H, I, R, d_G, st); break;
+    case 2: *status = launch_gram_dmma<2>(d_H, I, R, d_G, st); break;
+    case 3: *status = launch_gram_dmma<3>(d_H, I, R, d_G, st); break;
+    case 4: *status = launch_gram_dmma<4>(d_H, I, R, d_G, st); break;
+    case 5: *status = launch_gram_dmma<5>(d_H, I, R, d_G, st); break;
+    case 6: *status = launch_gram_dmma<6>(d_H, I, R, d_G, st); break;
+    case 7: *status = launch_gram_dmma<7>(d_H, I, R, d_G, st); break;
+    default: *status = launch_gram_dmma<8>(d_H, I, R, d_G, st); break;
+  }
+  return true;
+}
 
 bool admm_can_fuse_gram(int R, double tol) { return tol == 0.0 && R <= 32; }
 

@@ -367,6 +367,8 @@ cstf_status scale_rows_by_cols(double* d_H, int64_t I, int R, const double* d_la
 }
 
 cstf_status gram_raw(const double* d_H, int64_t I, int R, double* d_G, cudaStream_t st) {
+  cstf_status gs = CSTF_OK;
+  if (gram_dmma(d_H, I, R, d_G, st, &gs)) return gs;      // R <= 64: FP64 tensor path (admm.cu)
   const int nb = gram_blocks(I);
   const int nb4 = ((R + 3) & ~3) / 4;
   const int E = nb4 * (nb4 + 1) / 2 * 16;

@@ -206,6 +206,8 @@ struct AdmmArgs {
 cstf_status admm_run(const AdmmArgs& a, const cstf_comm* comm, cudaStream_t st,
                      cstf_admm_stats* stats, int* iters_out, int64_t* launches);
 bool admm_can_fuse_gram(int R, double tol);
+// G = H^T H on the DMMA path for R <= 64 (returns false if not applicable; *status = launch status)
+bool gram_dmma(const double* d_H, int64_t I, int R, double* d_G, cudaStream_t st, cstf_status* status);
 
 // f1 update schemes (HALS / MU), same row-wise shape as ADMM
 struct UpdArgs {

@@ -175,6 +175,25 @@ def test_mttkrp_deterministic(B):
     assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[1], outs[2])
 
 
+@pytest.mark.parametrize("dmma", ["1", "0"])
+@pytest.mark.parametrize("I,R", [(0, 8), (1, 1), (7, 5), (1000, 13), (100003, 32), (4097, 40), (250001, 64),
+                                 (999, 65)])
+def test_gram_paths(B, I, R, dmma, monkeypatch):
+    """cstf_gram on the DMMA path (R <= 64) and on the DFMA register-tile kernel, ragged
+    row counts and ranks, against the oracle's Gram; repeatable bit for bit."""
+    monkeypatch.setenv("CSTF_GRAM_DMMA", dmma)
+    H = datagen.uniform(9, 78, I * R).reshape(I, R) - 0.25
+    Hd = cu(H)
+    G = cu(np.full((R, R), np.nan))
+    B.cstf_gram(Hd, G)
+    first = host(G).copy()
+    B.cstf_gram(Hd, G)
+    assert np.array_equal(host(G), first)
+    want = oracle.gram(H) if I > 0 else np.zeros((R, R))
+    assert normwise(first, want) <= 1e-12 if I > 0 else np.array_equal(first, want)
+    assert np.array_equal(first, first.T)
+
+
 @pytest.mark.parametrize("I,R", [(1, 4), (1000, 8), (4099, 32), (777, 64), (300, 100), (5000, 3)])
 def test_gram_and_normalize(B, I, R):
     H = datagen.uniform(5, 77, I * R).reshape(I, R)

@@ -89,8 +89,7 @@ int comm_rank(const cstf_comm* c);
 // and sums the partials over kb in fixed order.  The factor rows of block kb are
 // staged in shared memory by the CTA that processes them.
 constexpr int kTileRows = 256;        // SMEM-slab blocks (opt-in CSTF_KBLOCK=1)
-constexpr int64_t kL2Rows = 65536;      // L2 blocks: 16 MB of factor rows at R = 32
-constexpr int64_t kL2Chunk = 256;       // MTTKRP chunk of an L2-blocked copy (dynamic order)
+constexpr int64_t kL2Rows = 100000;     // L2 blocks: 25.6 / 51.2 MB of factor rows at R = 32 / 64
 struct ModeStore {
   int64_t I = 0;            // rows of this mode (local rows when distributed)
   int64_t nnz = 0;          // nonzeros in this copy
@@ -112,6 +111,7 @@ struct ModeStore {
   // cached chunk boundaries of the MTTKRP work split (depend only on the store)
   mutable DevBuf clb, ccont;
   mutable int64_t cchunk = -1, cnchunks = 0;
+  mutable std::vector<int64_t> kp;   // L2-blocked copies: first nonzero of each block (host, cached)
 };
 inline int record_bytes(int N) { return ((4 * (N - 1) + 8) + 15) / 16 * 16; }
 

@@ -32,7 +32,9 @@ struct MArgs {
   const int64_t* rowptr;
   const char* rec;
   const double* F[7];   // factor of record slot q
-  int64_t I, nnz, chunk, nchunks;
+  int64_t I, nnz, chunk, nchunks;   // I: end row (absolute); nnz: nonzeros of this launch
+  int64_t pbase, rbase;             // first nonzero / first (virtual) row of this launch; a.M row 0 = rbase
+  int64_t cbase;                    // absolute index of chunk 0 (chunk c = [(cbase + c) chunk, ...) clipped)
   int R, recb, nother;
   const int64_t* lb;    // [nchunks+1] first row with rowptr >= start of chunk c (lb[nchunks] = I)
   const int32_t* cont;  // [nchunks] row continuing into chunk c from an earlier chunk, or -1
@@ -44,28 +46,34 @@ struct MArgs {
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
 };
 
+// Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
+// nonzero range: a launch over a batch of L2 blocks splits every row exactly where
+// one launch over all blocks would (same arithmetic, bit for bit).
 __device__ __forceinline__ int64_t chunk_begin(const MArgs& a, int64_t c) {
-  return a.wstart ? a.wstart[c] : c * a.chunk;
+  return a.wstart ? a.wstart[c] : max(a.pbase, (a.cbase + c) * a.chunk);
 }
 __device__ __forceinline__ int64_t chunk_end(const MArgs& a, int64_t c) {
-  return a.wstart ? a.wstart[c + 1] : min((c + 1) * a.chunk, a.nnz);
+  return a.wstart ? a.wstart[c + 1] : min((a.cbase + c + 1) * a.chunk, a.pbase + a.nnz);
 }
 
-__global__ void k_chunk_bounds(const int64_t* __restrict__ rowptr, int64_t I, int64_t nnz,
-                               int64_t chunk, int64_t nchunks, const int64_t* __restrict__ wstart,
-                               int64_t* __restrict__ lb, int32_t* __restrict__ cont) {
+// Chunk c covers nonzeros [pbase + c chunk, ...) of rows [rbase, rend) (absolute
+// row and nonzero positions; a launch over a batch of L2 blocks uses a sub-range).
+__global__ void k_chunk_bounds(const int64_t* __restrict__ rowptr, int64_t rbase, int64_t rend, int64_t pbase,
+                               int64_t pend, int64_t chunk, int64_t cbase, int64_t nchunks,
+                               const int64_t* __restrict__ wstart, int64_t* __restrict__ lb,
+                               int32_t* __restrict__ cont) {
   for (int64_t c = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; c <= nchunks;
        c += (int64_t)gridDim.x * blockDim.x) {
-    if (c == nchunks) { lb[c] = I; continue; }
-    const int64_t p0 = wstart ? wstart[c] : c * chunk;
-    int64_t lo = 0, hi = I;          // lower_bound: first row r with rowptr[r] >= p0
+    if (c == nchunks) { lb[c] = rend; continue; }
+    const int64_t p0 = wstart ? wstart[c] : max(pbase, (cbase + c) * chunk);
+    int64_t lo = rbase, hi = rend;   // lower_bound: first row r with rowptr[r] >= p0
     while (lo < hi) {
       const int64_t mid = (lo + hi) >> 1;
       if (rowptr[mid] < p0) lo = mid + 1; else hi = mid;
     }
     lb[c] = lo;
     int32_t ct = -1;                 // the row containing p0 started before p0
-    if (p0 < nnz && lo > 0 && (lo == I || rowptr[lo] > p0)) ct = (int32_t)(lo - 1);
+    if (p0 < pend && lo > rbase && (lo == rend || rowptr[lo] > p0)) ct = (int32_t)(lo - 1);
     cont[c] = ct;
   }
 }
@@ -116,7 +124,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
           acc[s].y += __shfl_xor_sync(0xffffffffu, acc[s].y, off);
         }
       if (sg == 0) {
-        double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + r * (int64_t)R;
+        double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (r - a.rbase) * (int64_t)R;
 #pragma unroll
         for (int s = 0; s < VPL; s++) reinterpret_cast<double2*>(dst)[gl + s * G] = acc[s];
       }
@@ -284,7 +292,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
 #pragma unroll
         for (int s = 0; s < CPL; s++) acc[s] = fma(v, w[s], acc[s]);
       }
-      double* dst = (ct >= 0 && row == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + row * (int64_t)R;
+      double* dst = (ct >= 0 && row == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (row - a.rbase) * (int64_t)R;
 #pragma unroll
       for (int s = 0; s < CPL; s++)
         if (lane + 32 * s < R) dst[lane + 32 * s] = acc[s];
@@ -302,7 +310,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
 constexpr int kFixGroup = 16;
 
 __device__ __forceinline__ int64_t chunk_of(int64_t p, int64_t chunk, const int64_t* wstart, int64_t nchunks) {
-  if (!wstart) return p / chunk;
+  if (!wstart) return p / chunk;     // absolute chunk index (subtract the launch's cbase)
   int64_t lo = 0, hi = nchunks - 1;            // last chunk with wstart <= p
   while (lo < hi) {
     const int64_t mid = (lo + hi + 1) >> 1;
@@ -312,7 +320,7 @@ __device__ __forceinline__ int64_t chunk_of(int64_t p, int64_t chunk, const int6
 }
 
 __global__ void k_carry_groups(const int32_t* __restrict__ cont, int64_t nchunks, const int64_t* __restrict__ rowptr,
-                               int64_t chunk, const int64_t* __restrict__ wstart,
+                               int64_t chunk, const int64_t* __restrict__ wstart, int64_t cbase,
                                const double* __restrict__ carry, int R, double* __restrict__ gsum) {
   const int lane = threadIdx.x & 31;
   const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -320,9 +328,9 @@ __global__ void k_carry_groups(const int32_t* __restrict__ cont, int64_t nchunks
   for (int64_t c = warp0; c < nchunks; c += nwarps) {
     const int32_t h = cont[c];
     if (h < 0) continue;
-    const int64_t c0 = chunk_of(rowptr[h], chunk, wstart, nchunks) + 1;
+    const int64_t c0 = chunk_of(rowptr[h], chunk, wstart, nchunks) - cbase + 1;
     if ((c - c0) % kFixGroup != 0) continue;                // not a group leader
-    const int64_t cend = min(chunk_of(rowptr[h + 1] - 1, chunk, wstart, nchunks), c + kFixGroup - 1);
+    const int64_t cend = min(chunk_of(rowptr[h + 1] - 1, chunk, wstart, nchunks) - cbase, c + kFixGroup - 1);
     for (int col = lane; col < R; col += 32) {
       double s0 = 0.0, s1 = 0.0, s2 = 0.0, s3 = 0.0;
       int64_t cc = c;
@@ -339,7 +347,7 @@ __global__ void k_carry_groups(const int32_t* __restrict__ cont, int64_t nchunks
 }
 
 __global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks, const int64_t* __restrict__ rowptr,
-                              int64_t chunk, const int64_t* __restrict__ wstart,
+                              int64_t chunk, const int64_t* __restrict__ wstart, int64_t cbase, int64_t rbase,
                               const double* __restrict__ gsum, int R, double* __restrict__ M) {
   const int lane = threadIdx.x & 31;
   const int64_t warp0 = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
@@ -347,22 +355,24 @@ __global__ void k_carry_fixup(const int32_t* __restrict__ cont, int64_t nchunks,
   for (int64_t c = warp0; c < nchunks; c += nwarps) {
     const int32_t h = cont[c];
     if (h < 0 || (c > 0 && cont[c - 1] == h)) continue;     // run starts only
-    const int64_t cend = chunk_of(rowptr[h + 1] - 1, chunk, wstart, nchunks);
+    const int64_t cend = chunk_of(rowptr[h + 1] - 1, chunk, wstart, nchunks) - cbase;
     for (int col = lane; col < R; col += 32) {
       double s = 0.0;
       for (int64_t cc = c; cc <= cend; cc += kFixGroup) s += gsum[cc * R + col];
-      M[(int64_t)h * R + col] += s;
+      M[((int64_t)h - rbase) * R + col] += s;
     }
   }
 }
 
-// M[i, :] = sum over blocks kb (in order) of the partial rows P[kb * I + i, :]
+// M[i, :] = sum over blocks kb (in order) of the partial rows P[kb * I + i, :]; with
+// acc, M is the running sum of earlier blocks (a batch of blocks continues it:
+// the same summation order as one pass over all blocks)
 __global__ void k_reduce_blocks(const double* __restrict__ Pv, int64_t I, int64_t nblk, int R,
-                                double* __restrict__ M) {
+                                double* __restrict__ M, int acc) {
   const int64_t n = I * R;
   for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n;
        x += (int64_t)gridDim.x * blockDim.x) {
-    double s = 0.0;
+    double s = acc ? M[x] : 0.0;
     for (int64_t kb = 0; kb < nblk; kb++) s += Pv[kb * n + x];
     M[x] = s;
   }
@@ -385,7 +395,7 @@ template <int NOTHER, int RECB>
 bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl) {
   // short rows (few nonzeros per row): row flushes dominate and latency hiding
   // needs more warps -> the 4-CTA/SM register budget; long rows -> 2 CTAs/SM
-  const bool short_rows = a.nnz < 64 * a.I;
+  const bool short_rows = a.nnz < 64 * (a.I - a.rbase);
   if (tiled) {
     switch (a.R) {     // slab = 256 rows x R doubles: 2 KB .. 128 KB
       case 8: return launch_tiled_r<NOTHER, RECB, 8>(a, grid, st);
@@ -492,6 +502,105 @@ cstf_status tiled_split(const ModeStore& ms, cudaStream_t st) {
   return CSTF_OK;
 }
 
+// L2-blocked copy: nonzeros ordered by (block of the
+// blocked factor's row, output row, ...).  Blocks are processed in batches whose
+// partial rows fit a workspace budget -- a quarter of the device memory, a
+// function of the device and the problem only, so results are deterministic
+// (CSTF_L2_BATCH_BYTES overrides; halved only if the allocation fails).  Every
+// batch is one launch over its own nonzero range with chunks taken from a global
+// counter in copy order, so the nonzeros in flight touch a narrow slice of the
+// blocked factor (its L2-resident slab); its partials continue the running sum of
+// M in block order.
+cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, double* d_M, cudaStream_t st,
+                              int64_t* nl) {
+  const DeviceInfo& di = device_info();
+  Workspace& w = ws();
+  const int64_t I = ms.I, nblk = ms.nblk, nnz = ms.nnz;
+  if ((int64_t)ms.kp.size() != nblk + 1) {           // block boundaries (host copy, cached)
+    CSTF_TRY(w.kbptr.ensure((size_t)(nblk + 1) * 8));
+    k_kb_offsets<<<(int)((nblk + 256) / 256), 256, 0, st>>>(ms.rowptr.as<int64_t>(), I, nblk, w.kbptr.as<int64_t>());
+    CSTF_LAUNCHED();
+    (*nl)++;
+    ms.kp.resize((size_t)nblk + 1);
+    CSTF_CUDA(cudaMemcpyAsync(ms.kp.data(), w.kbptr.p, ms.kp.size() * 8, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  const size_t per_block = (size_t)I * R * 8;
+  size_t budget = 0;
+  if (const char* be = getenv("CSTF_L2_BATCH_BYTES")) {
+    budget = (size_t)atoll(be);
+  } else {
+    size_t fr = 0, tot = 0;
+    CSTF_CUDA(cudaMemGetInfo(&fr, &tot));
+    budget = tot / 4;
+  }
+  int64_t B = std::max<int64_t>(1, std::min<int64_t>(nblk, (int64_t)(budget / std::max<size_t>(per_block, 1))));
+  while (w.partial.ensure((size_t)B * per_block) != CSTF_OK) {
+    if (B == 1) return fail(CSTF_ERR_OUT_OF_MEMORY, "MTTKRP partial rows of one L2 block (set CSTF_L2_BLOCK=0)");
+    B = (B + 1) / 2;
+  }
+  const bool short_rows = nnz < 64 * ms.Ivirt;        // = launch_fast's CTA budget
+  const int ctas = di.sms * (short_rows ? 4 : 2);      // resident CTAs only
+  // chunk: the window in flight (resident warps x chunk) about half a block
+  int64_t chunk = (nnz / std::max<int64_t>(nblk, 1)) / (2 * (int64_t)ctas * kWarps);
+  chunk = std::min<int64_t>(1024, std::max<int64_t>(256, (chunk + 31) / 32 * 32));
+  if (const char* ce = getenv("CSTF_L2_CHUNK"))
+    if (atoll(ce) >= 32) chunk = (atoll(ce) + 31) / 32 * 32;
+  CSTF_TRY(w.queue.ensure(8));
+  double* part = w.partial.as<double>();
+  for (int64_t b0 = 0; b0 < nblk; b0 += B) {
+    const int64_t b1 = std::min(nblk, b0 + B);
+    const int64_t pbase = ms.kp[(size_t)b0], pend = ms.kp[(size_t)b1];
+    const int64_t rbase = b0 * I, rend = b1 * I;
+    const int64_t n = pend - pbase;
+    const int64_t cbase = pbase / chunk;
+    const int64_t nchunks = n > 0 ? (pend + chunk - 1) / chunk - cbase : 1;
+    CSTF_TRY(w.carry.ensure((size_t)nchunks * R * 8));
+    CSTF_TRY(w.gsum.ensure((size_t)nchunks * R * 8));
+    CSTF_TRY(w.lb.ensure((size_t)(nchunks + 1) * 8));
+    CSTF_TRY(w.cont.ensure((size_t)nchunks * 4));
+    const int gb = (int)std::min<int64_t>((nchunks + 1 + 255) / 256, (int64_t)di.sms * 8);
+    k_chunk_bounds<<<gb, 256, 0, st>>>(a.rowptr, rbase, rend, pbase, pend, chunk, cbase, nchunks, nullptr,
+                                        w.lb.as<int64_t>(), w.cont.as<int32_t>());
+    CSTF_LAUNCHED();
+    a.pbase = pbase;
+    a.cbase = cbase;
+    a.rbase = rbase;
+    a.I = rend;
+    a.nnz = n;
+    a.chunk = chunk;
+    a.nchunks = nchunks;
+    a.lb = w.lb.as<int64_t>();
+    a.cont = w.cont.as<int32_t>();
+    a.M = part;
+    a.carry = w.carry.as<double>();
+    a.queue = nullptr;
+    if (nchunks > 1) {
+      CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
+      a.queue = w.queue.as<unsigned long long>();
+    }
+    const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)ctas);
+    CSTF_TRY(launch_main(a, grid, grid, st, gl));
+    *nl += 2;
+    if (nchunks > 1) {
+      const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);
+      k_carry_groups<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, nullptr, cbase, a.carry, R,
+                                        w.gsum.as<double>());
+      CSTF_LAUNCHED();
+      k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, nullptr, cbase, rbase, w.gsum.as<double>(),
+                                       R, part);
+      CSTF_LAUNCHED();
+      *nl += 2;
+    }
+    const int64_t nm = I * R;
+    const int g = (int)std::min<int64_t>((nm + 255) / 256, (int64_t)di.sms * 16);
+    k_reduce_blocks<<<g, 256, 0, st>>>(part, I, b1 - b0, R, d_M, b0 > 0 ? 1 : 0);
+    CSTF_LAUNCHED();
+    (*nl)++;
+  }
+  return CSTF_OK;
+}
+
 }  // namespace
 
 cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d_factors,
@@ -501,12 +610,41 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   const DeviceInfo& di = device_info();
   const int64_t nnz = ms.nnz;
   Workspace& w = ws();
+  if (ms.I == 0) return CSTF_OK;
   MArgs a;
   a.wstart = nullptr;
   a.ckb = nullptr;
   a.queue = nullptr;
+  a.pbase = 0;
+  a.cbase = 0;
+  a.rbase = 0;
+  a.rowptr = ms.rowptr.as<int64_t>();
+  a.rec = ms.rec.as<char>();
+  a.recb = ms.recb;
+  a.nother = N - 1;
+  for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
+  a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor
+  a.R = R;
+  // Lanes per factor row: 8 lanes x 32 B (4 nonzeros per warp step) when the gathered
+  // factors are L2-resident -- more nonzeros per load instruction, so adjacent
+  // fiber nonzeros share L1 wavefronts (NELL-2 1.80 -> 1.63 ms per mode); the
+  // default 16 lanes x 16 B when they stream from HBM (Delicious, Amazon: no gain
+  // or a loss).  CSTF_MTTKRP_G forces a value (experiments).
+  int gl = 0;
+  {
+    int64_t gbytes = 0;
+    for (int q = 0; q < N - 1; q++) gbytes += X->dims[ms.other[q]] * (int64_t)R * 8;
+    if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
+    const char* ge = getenv("CSTF_MTTKRP_G");        // read per call (tests force both paths)
+    if (ge && (atoi(ge) == 0 || atoi(ge) == 8)) gl = atoi(ge);
+  }
+  int64_t nl = 0;
+  if (ms.tiled && !ms.slab) {
+    CSTF_TRY(mttkrp_l2_blocked(ms, a, R, gl, d_M, st, &nl));
+    if (launches) *launches += nl;
+    return CSTF_OK;
+  }
   int64_t chunk = 0, nchunks = 0;
-  const bool l2blk = ms.tiled && !ms.slab;
   if (ms.tiled && ms.slab) {
     CSTF_TRY(tiled_split(ms, st));
     nchunks = ms.nwchunks;
@@ -515,14 +653,10 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   } else {
     // chunk: ~4 chunks per resident warp, multiple of 32, in [256, 8192]
     const int64_t resident = (int64_t)di.sms * 8 * kWarps;
-    chunk = (nnz + resident * 4 - 1) / (resident * 4);   // (virtual rows when L2-blocked)
+    chunk = (nnz + resident * 4 - 1) / (resident * 4);
     chunk = ((chunk + 31) / 32) * 32;
     if (chunk < 256) chunk = 256;
     if (chunk > 8192) chunk = 8192;
-    if (l2blk) {     // dynamic order: the window in flight = resident warps x chunk nonzeros
-      const char* ce = getenv("CSTF_L2_CHUNK");
-      chunk = ce && atoll(ce) >= 32 ? (atoll(ce) + 31) / 32 * 32 : kL2Chunk;
-    }
     nchunks = nnz > 0 ? (nnz + chunk - 1) / chunk : 1;
   }
   CSTF_TRY(w.carry.ensure((size_t)nchunks * R * 8));
@@ -537,69 +671,40 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     CSTF_TRY(w.partial.ensure((size_t)ms.Ivirt * R * 8));
     out = w.partial.as<double>();
   }
-  a.rowptr = ms.rowptr.as<int64_t>();
-  a.rec = ms.rec.as<char>();
-  a.recb = ms.recb;
-  a.nother = N - 1;
-  for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
-  a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor
   a.I = ms.Ivirt;
   a.nnz = nnz;
   a.chunk = chunk;
   a.nchunks = nchunks;
-  a.R = R;
   a.lb = ms.clb.as<int64_t>();
   a.cont = ms.ccont.as<int32_t>();
   a.M = out;
   a.carry = w.carry.as<double>();
-  if (ms.I == 0) return CSTF_OK;
-  int64_t nl = 0;
   if (fresh) {
     const int g = (int)std::min<int64_t>((nchunks + 1 + 255) / 256, (int64_t)di.sms * 8);
-    k_chunk_bounds<<<g, 256, 0, st>>>(a.rowptr, ms.Ivirt, nnz, chunk, nchunks, a.wstart, ms.clb.as<int64_t>(),
-                                       ms.ccont.as<int32_t>());
+    k_chunk_bounds<<<g, 256, 0, st>>>(a.rowptr, 0, ms.Ivirt, 0, nnz, chunk, 0, nchunks, a.wstart,
+                                       ms.clb.as<int64_t>(), ms.ccont.as<int32_t>());
     CSTF_LAUNCHED();
     nl++;
     ms.cchunk = chunk;
     ms.cnchunks = nchunks;
   }
-  int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
-  if (l2blk && nchunks > 1) {
-    CSTF_TRY(w.queue.ensure(8));
-    CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
-    a.queue = w.queue.as<unsigned long long>();
-    const bool short_rows = nnz < 64 * ms.Ivirt;        // = launch_fast's CTA budget
-    grid = (int)std::min<int64_t>(grid, (int64_t)di.sms * (short_rows ? 4 : 2));   // resident CTAs only
-  }
+  const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)di.sms * 8);
   const int tgrid = (int)std::min<int64_t>(std::max<int64_t>(ms.nctachunks, 1), (int64_t)di.sms * 2);
-  // (a.ckb is set only for SMEM-slab copies; L2-blocked copies run the flat kernel on virtual rows)
-  // Lanes per factor row: 8 lanes x 32 B (4 nonzeros per warp step) when the gathered
-  // factors are L2-resident -- more nonzeros per load instruction, so adjacent
-  // fiber nonzeros share L1 wavefronts (NELL-2 1.80 -> 1.63 ms per mode); the
-  // default 16 lanes x 16 B when they stream from HBM (Delicious, Amazon: no gain
-  // or a loss).  CSTF_MTTKRP_G forces a value (experiments).
-  int gl = 0;
-  {
-    int64_t gbytes = 0;
-    for (int q = 0; q < N - 1; q++) gbytes += X->dims[ms.other[q]] * (int64_t)R * 8;
-    if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
-    const char* ge = getenv("CSTF_MTTKRP_G");        // read per call (tests force both paths)
-    if (ge && (atoi(ge) == 0 || atoi(ge) == 8)) gl = atoi(ge);
-  }
   CSTF_TRY(launch_main(a, grid, tgrid, st, gl));
   nl++;
   if (nchunks > 1) {
     const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);
-    k_carry_groups<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, a.carry, R, w.gsum.as<double>());
+    k_carry_groups<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, 0, a.carry, R,
+                                      w.gsum.as<double>());
     CSTF_LAUNCHED();
-    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, w.gsum.as<double>(), R, out);
+    k_carry_fixup<<<g, 256, 0, st>>>(a.cont, nchunks, a.rowptr, chunk, a.wstart, 0, 0, w.gsum.as<double>(), R, out);
     CSTF_LAUNCHED();
     nl += 2;
   }
   if (ms.tiled) {
     const int64_t n = ms.I * R;
     const int g = (int)std::min<int64_t>((n + 255) / 256, (int64_t)di.sms * 16);
-    k_reduce_blocks<<<g, 256, 0, st>>>(out, ms.I, ms.nblk, R, d_M);
+    k_reduce_blocks<<<g, 256, 0, st>>>(out, ms.I, ms.nblk, R, d_M, 0);
     CSTF_LAUNCHED();
     nl++;
   }

@@ -580,22 +580,29 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
         ms.tiled = ms.slab = true; ms.blk_rows = kTileRows; ms.nblk = nb; ms.tslot = N - 2;
       }
     } else if (N >= 3 && !(getenv("CSTF_L2_BLOCK") && atoi(getenv("CSTF_L2_BLOCK")) == 0)) {
-      // Default: only where the partial rows are nearly free -- a short output
-      // mode (nblk * I_n <= nnz / 64) against a factor that does not fit L2 even
-      // at R = 32 (Delicious mode 4: 13.1 -> 10.7 ms).  CSTF_L2_BLOCK_ROWS /
-      // CSTF_L2_BLOCK_MAXROWS widen it (experiments: slower on long output
-      // modes -- the partial rows cost what the L2 hits save).
+      // Default: block by the largest other factor t when it does not fit L2 even at
+      // R = 32 (I_t * 256 B > L2) and the partial rows pay for themselves:
+      //  * short output mode, partial rows nearly free: nblk * I_n <= nnz / 64
+      //    (Delicious mode 4: 13.1 -> 10.3 ms), or
+      //  * long rows: >= 8 nonzeros per (row, block) on average, nnz >= 8 nblk I_n
+      //    (Amazon: 678 -> ~569 ms of MTTKRP per outer iteration).
+      // Delicious modes 1-3 satisfy neither (blocking them measured slower).
+      // CSTF_L2_BLOCK_ROWS / CSTF_L2_BLOCK_MAXROWS force it (tests, experiments).
       const char* ov = getenv("CSTF_L2_BLOCK_ROWS");
       const bool forced = ov != nullptr;
       const int64_t l2rows = ov && atoll(ov) > 0 ? atoll(ov) : kL2Rows;
       const int64_t maxv = getenv("CSTF_L2_BLOCK_MAXROWS") ? atoll(getenv("CSTF_L2_BLOCK_MAXROWS"))
-                                                          : (forced ? ((int64_t)16 << 20) : nout / 64);
-      for (int q = N - 2; q >= 0 && !ms.tiled; q--) {     // largest other factor first
+                                                          : ((int64_t)16 << 20);
+      for (int q = N - 2; q >= (forced ? 0 : N - 2) && !ms.tiled; q--) {     // largest other factor first
         const int tm = ms.other[q];
         const int64_t nb = (X->dims[tm] + l2rows - 1) / l2rows;
-        const bool big = forced || X->dims[tm] * 256 > (int64_t)device_info().l2;
-        if (big && X->dims[tm] > 2 * l2rows && nb * ms.I <= maxv && nb * ms.I < ((int64_t)1 << 31) &&
-            nout >= 4 * nb * ms.I) {
+        bool ok = X->dims[tm] > 2 * l2rows && nb * ms.I < ((int64_t)1 << 31) && nout >= 4 * nb * ms.I;
+        if (forced)
+          ok = ok && nb * ms.I <= maxv;
+        else
+          ok = ok && X->dims[tm] * 256 > (int64_t)device_info().l2 &&
+               (nb * ms.I * 64 <= nout || nout >= 8 * nb * ms.I);
+        if (ok) {
           ms.tiled = true; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = q; t = tm;
         }
       }

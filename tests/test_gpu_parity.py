@@ -495,6 +495,11 @@ def test_mttkrp_l2_blocked_copies(B, R, monkeypatch):
         M = cu(np.full((dims[n], R), np.nan))
         B.cstf_mttkrp(X, n, Fd, M)
         assert normwise(host(M), oracle.mttkrp(ref, n, F)) <= TOL, n
+        monkeypatch.setenv("CSTF_L2_BATCH_BYTES", "1")        # one block per batch
+        M1 = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M1)
+        monkeypatch.delenv("CSTF_L2_BATCH_BYTES")
+        assert normwise(host(M1), host(M)) <= TOL, n
     lam = cu(np.zeros(R))
     gpu = B.cstf_factorize(X, Fd, lam, B.make_opts(R, outer_iters=3, tol=1e-2))
     orc = oracle.factorize(ref, F, outer_iters=3, tol=1e-2)
@@ -530,6 +535,35 @@ def test_mttkrp_l2_blocked_default(B, monkeypatch):
         Mp = cu(np.full((dims[n], R), np.nan))
         B.cstf_mttkrp(Xp, n, Fd, Mp)
         assert normwise(first, host(Mp)) <= TOL, n
+
+
+@pytest.mark.parametrize("R", [16, 32])
+def test_mttkrp_l2_blocked_long_rows_batches(B, R, monkeypatch):
+    """Default L2 blocking of a long-row output mode (the Amazon case: >= 8 nonzeros per
+    (row, block)); blocks processed in batches of any size (forced small budgets)
+    match the oracle, and a fixed budget is bitwise repeatable."""
+    dims = (20_000, 600_000, 30)
+    idx, vals = datagen.coo(dims, (2, 2, 3), 5_000_000, 31)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    nblk, rows, bm = X.layout(0)
+    assert bm == 1 and nblk == -(-dims[1] // rows) and nblk > 1
+    ref = oracle.coalesce(dims, idx, vals)
+    F = datagen.init_factors(dims, R, 6)
+    Fd = [cu(f) for f in F]
+    outs = []
+    for budget in (None, 1, 3 * dims[0] * R * 8):
+        if budget is None:
+            monkeypatch.delenv("CSTF_L2_BATCH_BYTES", raising=False)
+        else:
+            monkeypatch.setenv("CSTF_L2_BATCH_BYTES", str(budget))
+        M = cu(np.full((dims[0], R), np.nan))
+        B.cstf_mttkrp(X, 0, Fd, M)
+        outs.append(host(M).copy())
+        B.cstf_mttkrp(X, 0, Fd, M)
+        assert np.array_equal(host(M), outs[-1])
+    want = oracle.mttkrp(ref, 0, F)
+    for o in outs:
+        assert normwise(o, want) <= TOL
 
 
 def test_factorize_bitwise_deterministic(B):

@@ -564,6 +564,14 @@ def test_mttkrp_l2_blocked_long_rows_batches(B, R, monkeypatch):
     want = oracle.mttkrp(ref, 0, F)
     for o in outs:
         assert normwise(o, want) <= TOL
+    # one launch per block with a persisting L2 window on its slab (forced at this size)
+    monkeypatch.delenv("CSTF_L2_BATCH_BYTES", raising=False)
+    monkeypatch.setenv("CSTF_L2_PERSIST", str(32 << 20))
+    M = cu(np.full((dims[0], R), np.nan))
+    B.cstf_mttkrp(X, 0, Fd, M)
+    first = host(M).copy()
+    B.cstf_mttkrp(X, 0, Fd, M)
+    assert np.array_equal(host(M), first) and normwise(first, want) <= TOL
 
 
 def test_factorize_bitwise_deterministic(B):

@@ -564,8 +564,12 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     persist = std::min<size_t>(persist, (size_t)std::max(maxp, 0));
     static thread_local size_t set_for[64] = {0};
     if (persist && set_for[di.device & 63] != persist) {
-      CSTF_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, persist));
-      set_for[di.device & 63] = persist;
+      if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, persist) == cudaSuccess) {
+        set_for[di.device & 63] = persist;
+      } else {                    // not available (e.g. MIG): plain launches, no error
+        cudaGetLastError();
+        persist = 0;
+      }
     }
   }
   for (int64_t b0 = 0; b0 < nblk; b0 += B) {
@@ -612,7 +616,7 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
         v.accessPolicyWindow.hitRatio = std::min(1.0f, (float)persist / (float)std::max<size_t>(v.accessPolicyWindow.num_bytes, 1));
         v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
         v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-        CSTF_CUDA(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v));
+        if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v) != cudaSuccess) cudaGetLastError();
       }
       const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)ctas);
       CSTF_TRY(launch_main(a, grid, grid, st, gl));
@@ -634,11 +638,11 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     CSTF_LAUNCHED();
     (*nl)++;
   }
-  if (persist) {
+  if (persist) {                  // drop the window and release the persisting lines
     cudaStreamAttrValue v = {};
     v.accessPolicyWindow.num_bytes = 0;
-    CSTF_CUDA(cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v));
-    CSTF_CUDA(cudaCtxResetPersistingL2Cache());
+    if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v) != cudaSuccess) cudaGetLastError();
+    if (cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
   }
   return CSTF_OK;
 }

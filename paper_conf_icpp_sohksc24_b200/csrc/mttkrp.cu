@@ -638,10 +638,13 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     CSTF_LAUNCHED();
     (*nl)++;
   }
-  if (persist) {                  // drop the window and release the persisting lines
+  if (persist) {
+    // drop the window; once the launches have run, release the persisting lines (the
+    // reset is not stream-ordered) so later kernels get the whole L2 back
     cudaStreamAttrValue v = {};
     v.accessPolicyWindow.num_bytes = 0;
     if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v) != cudaSuccess) cudaGetLastError();
+    CSTF_CUDA(cudaStreamSynchronize(st));
     if (cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
   }
   return CSTF_OK;

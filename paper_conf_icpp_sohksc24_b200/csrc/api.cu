@@ -36,7 +36,9 @@ bool rank_ok(int R) { return R >= 1 && R <= 128; }
 
 // Device-side scratch of one factorize / admm_update call, cached per device.
 struct DriverWs {
-  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8], S;
+  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8], S, stage;
+  cudaStream_t copy = nullptr;   // host <-> device factor transfers of cstf_factorize_host
+  cudaEvent_t ev_in[8] = {nullptr}, ev_out[8] = {nullptr};
   // distributed: all internal factor replicas in one allocation, mapped by the
   // other ranks through CUDA IPC (NVLink peer memory) for the fused all-gather
   DevBuf facall, xchg;
@@ -57,6 +59,11 @@ DriverWs& dws() {
     cudaStreamCreateWithFlags(&r.side, cudaStreamNonBlocking);
     cudaEventCreateWithFlags(&r.fork, cudaEventDisableTiming);
     cudaEventCreateWithFlags(&r.join, cudaEventDisableTiming);
+    cudaStreamCreateWithFlags(&r.copy, cudaStreamNonBlocking);
+    for (int n = 0; n < 8; n++) {
+      cudaEventCreateWithFlags(&r.ev_in[n], cudaEventDisableTiming);
+      cudaEventCreateWithFlags(&r.ev_out[n], cudaEventDisableTiming);
+    }
   }
   return r;
 }
@@ -157,9 +164,20 @@ struct PhaseTimer {
   }
 };
 
+// Host I/O of cstf_factorize_host overlapped with the computation (single GPU):
+// host_in[n] -> d_factors[n] on the copy stream, in the order the first outer
+// iteration needs them (factor 0 only before the first ADMM update); with a
+// fixed number of outer iterations, each final factor is normalised into a
+// staging copy right after its last update and copied to host_out[n] while the
+// later modes compute.
+struct HostIO {
+  double* const* in = nullptr;
+  double* const* out = nullptr;
+};
+
 cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_comm* comm,
                            double* const* d_factors, double* d_lambda, cstf_report* rep,
-                           cudaStream_t st) {
+                           cudaStream_t st, const HostIO* hio = nullptr) {
   const int N = X->N;
   const int R = o->R;
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
@@ -227,15 +245,40 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   }
   CSTF_CUDA(cudaMemsetAsync(flag, 0, 4, st));
   CSTF_CUDA(cudaMemsetAsync(w.U.p, 0, (size_t)Usum * 8, st));
+  const bool hin = hio && hio->in && !dist;
+  const bool hout = hio && hio->out && !dist && o->fit_tol <= 0.0;
+  if (hin) {                         // factors 1..N-1 first, factor 0 last (needed only by ADMM(0))
+    CSTF_CUDA(cudaEventRecord(w.fork, st));
+    CSTF_CUDA(cudaStreamWaitEvent(w.copy, w.fork, 0));
+    for (int k = 1; k <= N; k++) {
+      const int n = k % N;
+      CSTF_CUDA(cudaMemcpyAsync(fac[n], hio->in[n], (size_t)Ifull[n] * R * 8, cudaMemcpyHostToDevice, w.copy));
+      CSTF_CUDA(cudaEventRecord(w.ev_in[n], w.copy));
+    }
+  }
   // init (Alg. 1 l.1-5; readings D6): normalise, lambda = 1, G = H^T H
-  for (int n = 0; n < N; n++) {      // factors are replicated: redundant, no communication
+  auto init_factor = [&](int n) -> cstf_status {
     double* Gn = G + (size_t)n * R * R;
+    if (hin) CSTF_CUDA(cudaStreamWaitEvent(st, w.ev_in[n], 0));
     CSTF_TRY(gram_raw(fac[n], Ifull[n], R, Gn, st));
     if (o->normalize_init) CSTF_TRY(normalize_from_gram(fac[n], Ifull[n], R, Gn, lam + n * R, st));
-    CSTF_TRY(fill(lam + n * R, R, 1.0, st));
+    return fill(lam + n * R, R, 1.0, st);
+  };
+  for (int n = 0; n < N; n++) {      // factors are replicated: redundant, no communication
+    if (hin && n == 0) {             // deferred: after MTTKRP(0) is queued
+      CSTF_TRY(fill(lam, R, 1.0, st));
+      continue;
+    }
+    CSTF_TRY(init_factor(n));
   }
   if (peers) {   // no rank may peer-store into a replica another rank is still initialising / reading
     CSTF_TRY(comm_allreduce_f64(comm, w.xchg.as<double>(), 1, st));
+  }
+  std::vector<int64_t> stage_off(N, 0);
+  if (hout) {
+    int64_t so = 0;
+    for (int n = 0; n < N; n++) { stage_off[n] = so; so += Ifull[n] * R; }
+    CSTF_TRY(w.stage.ensure((size_t)so * 8));
   }
   PhaseTimer tm;
   tm.on = o->timing != 0;
@@ -273,6 +316,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       // a2: MTTKRP of the raw factors (MTTKRP phase = both, overlapped)
       tm.begin(n, CSTF_PHASE_MTTKRP);
       CSTF_TRY(mttkrp(X, n, R, fac.data(), M, st, nullptr));
+      if (hin && t == 0 && n == 0) CSTF_TRY(init_factor(0));   // its copy overlapped MTTKRP(0)
       CSTF_CUDA(cudaStreamWaitEvent(st, w.join, 0));
       tm.end(n, CSTF_PHASE_MTTKRP);
       // a5: ADMM on M diag(mscale); warm start H_raw (D4) or the normalised H (literal)
@@ -331,6 +375,14 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       CSTF_TRY(comm_allreduce_f64(comm, Gn, (size_t)R * R, st));
       CSTF_TRY(gram_to_lambda(Gn, R, lam + n * R, st));
       tm.end(n, CSTF_PHASE_NORMALIZE);
+      if (hout && t == o->outer_iters - 1) {   // final factor n: normalised copy to the host now
+        double* sn = w.stage.as<double>() + stage_off[n];
+        CSTF_CUDA(cudaMemcpyAsync(sn, fac[n], (size_t)Ifull[n] * R * 8, cudaMemcpyDeviceToDevice, st));
+        CSTF_TRY(scale_rows_by_cols(sn, Ifull[n], R, lam + n * R, 1, st));
+        CSTF_CUDA(cudaEventRecord(w.ev_out[n], st));
+        CSTF_CUDA(cudaStreamWaitEvent(w.copy, w.ev_out[n], 0));
+        CSTF_CUDA(cudaMemcpyAsync(hio->out[n], sn, (size_t)Ifull[n] * R * 8, cudaMemcpyDeviceToHost, w.copy));
+      }
     }
     // a8: fit of [[lambda^(N); H]]: inner product of M'(N) diag(mscale) with H_raw(N)
     tm.begin(N - 1, CSTF_PHASE_NORMALIZE);
@@ -356,7 +408,11 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   }
   if (d_lambda)
     CSTF_CUDA(cudaMemcpyAsync(d_lambda, lam + (N - 1) * R, (size_t)R * 8, cudaMemcpyDeviceToDevice, st));
+  if (hio && hio->out && !hout)      // no overlap possible (fit_tol or distributed): copy at the end
+    for (int n = 0; n < N; n++)
+      CSTF_CUDA(cudaMemcpyAsync(hio->out[n], d_factors[n], (size_t)X->dims[n] * R * 8, cudaMemcpyDeviceToHost, st));
   CSTF_CUDA(cudaStreamSynchronize(st));
+  if (hin || hout) CSTF_CUDA(cudaStreamSynchronize(w.copy));
   return CSTF_OK;
 }
 
@@ -518,16 +574,19 @@ cstf_status cstf_factorize_host(const cstf_tensor* X, const cstf_opts* opts, con
   CSTF_TRY(w.hostfac.ensure((size_t)(tot + R) * 8));
   std::vector<double*> d(N);
   int64_t off = 0;
+  const bool dist = X->partitioned;
   for (int n = 0; n < N; n++) {
     if (!host_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "host factor pointer is NULL");
     d[n] = w.hostfac.as<double>() + off;
-    CSTF_CUDA(cudaMemcpyAsync(d[n], host_factors[n], (size_t)X->dims[n] * R * 8, cudaMemcpyHostToDevice, st));
+    if (dist)                        // (the partitioned path relabels from device copies first)
+      CSTF_CUDA(cudaMemcpyAsync(d[n], host_factors[n], (size_t)X->dims[n] * R * 8, cudaMemcpyHostToDevice, st));
     off += X->dims[n] * R;
   }
   double* d_lam = w.hostfac.as<double>() + off;
-  CSTF_TRY(factorize_impl(X, opts, comm, d.data(), d_lam, report, st));
-  for (int n = 0; n < N; n++)
-    CSTF_CUDA(cudaMemcpyAsync(host_factors[n], d[n], (size_t)X->dims[n] * R * 8, cudaMemcpyDeviceToHost, st));
+  HostIO io;
+  io.in = dist ? nullptr : host_factors;
+  io.out = host_factors;
+  CSTF_TRY(factorize_impl(X, opts, comm, d.data(), d_lam, report, st, &io));
   if (host_lambda) CSTF_CUDA(cudaMemcpyAsync(host_lambda, d_lam, (size_t)R * 8, cudaMemcpyDeviceToHost, st));
   CSTF_CUDA(cudaStreamSynchronize(st));
   return CSTF_OK;

@@ -370,22 +370,31 @@ def test_factorize_fixed_iterations_protocol(B):
         assert normwise(a, b) <= 1e-6
 
 
-def test_factorize_host_matches_device(B):
+@pytest.mark.parametrize("R,outer,tol,fit_tol,pinned", [(8, 3, 1e-2, 0.0, False), (32, 4, 0.0, 0.0, True),
+                                                       (16, 3, 0.0, 1e-12, True), (5, 1, 0.0, 0.0, False)])
+def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned):
+    """The host-buffer path (factor copies overlapped with the computation: factor 0
+    copied in during MTTKRP(0), each final factor copied out after its last update)
+    gives the bits of the device path."""
     c = datagen.CONFIGS["enron"].scaled(60, nnz_factor=2000)
     idx, vals = c.generate()
     X = B.cstf_tensor_load_coo(c.dims, idx, vals)
-    start = datagen.init_factors(c.dims, 8, 1)
-    opts = B.make_opts(8, outer_iters=3, tol=1e-2)
+    start = datagen.init_factors(c.dims, R, 1)
+    opts = B.make_opts(R, outer_iters=outer, tol=tol, fit_tol=fit_tol)
     F = [cu(f) for f in start]
-    lam = cu(np.zeros(8))
+    lam = cu(np.zeros(R))
     g1 = B.cstf_factorize(X, F, lam, opts)
-    hf = [f.copy() for f in start]
-    hl = np.zeros(8)
+    if pinned:
+        hf = [torch.from_numpy(f.copy()).pin_memory() for f in start]
+        hl = torch.zeros(R, dtype=torch.float64).pin_memory()
+    else:
+        hf = [f.copy() for f in start]
+        hl = np.zeros(R)
     g2 = B.cstf_factorize_host(X, hf, hl, opts)
     assert np.array_equal(g1["fit"], g2["fit"])
     for a, b in zip(hf, F):
-        assert np.array_equal(a, host(b))
-    assert np.array_equal(hl, host(lam))
+        assert np.array_equal(np.asarray(a), host(b))
+    assert np.array_equal(np.asarray(hl), host(lam))
 
 
 @pytest.mark.parametrize("R", [8, 32, 5, 64])

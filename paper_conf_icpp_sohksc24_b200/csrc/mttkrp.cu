@@ -673,7 +673,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.nother = N - 1;
   for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
   a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor
-  a.It_blk = X->dims[ms.other[ms.tslot]];
+  a.It_blk = X->partitioned ? (int64_t)X->nranks * X->rows_per_rank[ms.other[ms.tslot]] : X->dims[ms.other[ms.tslot]];
   a.R = R;
   // Lanes per factor row: 8 lanes x 32 B (4 nonzeros per warp step) when the gathered
   // factors are L2-resident -- more nonzeros per load instruction, so adjacent

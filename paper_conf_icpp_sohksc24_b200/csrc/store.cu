@@ -325,6 +325,38 @@ cstf_status build_rowptr(const int32_t* d_key, int64_t n, int64_t I, DevBuf& row
   return CSTF_OK;
 }
 
+// L2-block decision for a mode copy with `nloc` nonzeros over `Iloc` output rows;
+// Ioth[q] = rows of the factor gathered through record slot q (slots by increasing
+// length).  Sets ms.tiled / blk_rows / nblk / tslot (L2 blocks, not SMEM slabs).
+//  Default: block by the largest other factor t when it does not fit L2 even at
+//  R = 32 (I_t * 256 B > L2) and the partial rows pay for themselves:
+//   * short output mode, partial rows nearly free: nblk * I_n <= nnz / 64
+//     (Delicious mode 4: 13.1 -> 10.3 ms), or
+//   * long rows: >= 8 nonzeros per (row, block) on average, nnz >= 8 nblk I_n
+//     (Amazon: 678 -> ~569 ms of MTTKRP per outer iteration).
+//  Delicious modes 1-3 satisfy neither (blocking them measured slower).
+//  CSTF_L2_BLOCK_ROWS / CSTF_L2_BLOCK_MAXROWS force it (tests, experiments).
+void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int64_t* Ioth) {
+  if (N < 3 || (getenv("CSTF_L2_BLOCK") && atoi(getenv("CSTF_L2_BLOCK")) == 0)) return;
+  const char* ov = getenv("CSTF_L2_BLOCK_ROWS");
+  const bool forced = ov != nullptr;
+  const int64_t l2rows = ov && atoll(ov) > 0 ? atoll(ov) : kL2Rows;
+  const int64_t maxv = getenv("CSTF_L2_BLOCK_MAXROWS") ? atoll(getenv("CSTF_L2_BLOCK_MAXROWS"))
+                                                      : ((int64_t)16 << 20);
+  for (int q = N - 2; q >= (forced ? 0 : N - 2) && !ms.tiled; q--) {     // largest other factor first
+    const int64_t It = Ioth[q];
+    const int64_t nb = (It + l2rows - 1) / l2rows;
+    bool ok = It > 2 * l2rows && nb * Iloc < ((int64_t)1 << 31) && nloc >= 4 * nb * Iloc;
+    if (forced)
+      ok = ok && nb * Iloc <= maxv;
+    else
+      ok = ok && It * 256 > (int64_t)device_info().l2 && (nb * Iloc * 64 <= nloc || nloc >= 8 * nb * Iloc);
+    if (ok) {
+      ms.tiled = true; ms.slab = false; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = q;
+    }
+  }
+}
+
 }  // namespace
 
 // Partitioned copies: rows of every mode are dealt to
@@ -418,17 +450,37 @@ cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int
                                                           vv.as<double>());
       CSTF_LAUNCHED();
     }
-    const int32_t* keys[8];
-    int64_t kd[8];
-    keys[0] = kk[0].as<int32_t>();
-    kd[0] = B;
+    // L2 blocks over the internal labels of the largest other factor (local rows B)
+    {
+      int64_t Ioth[7];
+      for (int q = 0; q < N - 1; q++) Ioth[q] = (int64_t)P * X->rows_per_rank[ms.other[q]];
+      ms.slab = false;
+      decide_l2_block(ms, N, ns, B, Ioth);
+      ms.Ivirt = ms.nblk * B;
+    }
+    const int32_t* keys[9];
+    int64_t kd[9];
+    int nk = 0;
+    DevBuf kbk, vrow;
+    if (ms.tiled) {
+      CSTF_TRY(kbk.alloc((size_t)ns * 4));
+      CSTF_TRY(vrow.alloc((size_t)ns * 4));
+      if (ns) {
+        k_block_keys<<<grid_for(ns), kThreads, 0, st>>>(kk[ms.tslot + 1].as<int32_t>(), kk[0].as<int32_t>(), ns, B,
+                                                        ms.blk_rows, kbk.as<int32_t>(), vrow.as<int32_t>());
+        CSTF_LAUNCHED();
+      }
+      keys[nk] = kbk.as<int32_t>(); kd[nk++] = ms.nblk;
+    }
+    keys[nk] = kk[0].as<int32_t>();
+    kd[nk++] = B;
     for (int q = 0; q < N - 1; q++) {
-      keys[q + 1] = kk[q + 1].as<int32_t>();
-      kd[q + 1] = (int64_t)P * X->rows_per_rank[ms.other[q]];
+      keys[nk] = kk[q + 1].as<int32_t>();
+      kd[nk++] = (int64_t)P * X->rows_per_rank[ms.other[q]];
     }
     DevBuf pm;
-    CSTF_TRY(lsd_sort(keys, kd, N, ns, pm, tmp, st));
-    CSTF_TRY(build_rowptr(kk[0].as<int32_t>(), ns, B, ms.rowptr, tmp, st));
+    CSTF_TRY(lsd_sort(keys, kd, nk, ns, pm, tmp, st));
+    CSTF_TRY(build_rowptr(ms.tiled ? vrow.as<int32_t>() : kk[0].as<int32_t>(), ns, ms.Ivirt, ms.rowptr, tmp, st));
     ms.nnz = ns;
     CSTF_TRY(ms.rec.alloc((size_t)ns * recb));
     RecArgs ra;
@@ -579,33 +631,11 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
       if (nb >= 2 && nb * ms.I <= ((int64_t)4 << 20) && nout >= 8 * nb * ms.I) {
         ms.tiled = ms.slab = true; ms.blk_rows = kTileRows; ms.nblk = nb; ms.tslot = N - 2;
       }
-    } else if (N >= 3 && !(getenv("CSTF_L2_BLOCK") && atoi(getenv("CSTF_L2_BLOCK")) == 0)) {
-      // Default: block by the largest other factor t when it does not fit L2 even at
-      // R = 32 (I_t * 256 B > L2) and the partial rows pay for themselves:
-      //  * short output mode, partial rows nearly free: nblk * I_n <= nnz / 64
-      //    (Delicious mode 4: 13.1 -> 10.3 ms), or
-      //  * long rows: >= 8 nonzeros per (row, block) on average, nnz >= 8 nblk I_n
-      //    (Amazon: 678 -> ~569 ms of MTTKRP per outer iteration).
-      // Delicious modes 1-3 satisfy neither (blocking them measured slower).
-      // CSTF_L2_BLOCK_ROWS / CSTF_L2_BLOCK_MAXROWS force it (tests, experiments).
-      const char* ov = getenv("CSTF_L2_BLOCK_ROWS");
-      const bool forced = ov != nullptr;
-      const int64_t l2rows = ov && atoll(ov) > 0 ? atoll(ov) : kL2Rows;
-      const int64_t maxv = getenv("CSTF_L2_BLOCK_MAXROWS") ? atoll(getenv("CSTF_L2_BLOCK_MAXROWS"))
-                                                          : ((int64_t)16 << 20);
-      for (int q = N - 2; q >= (forced ? 0 : N - 2) && !ms.tiled; q--) {     // largest other factor first
-        const int tm = ms.other[q];
-        const int64_t nb = (X->dims[tm] + l2rows - 1) / l2rows;
-        bool ok = X->dims[tm] > 2 * l2rows && nb * ms.I < ((int64_t)1 << 31) && nout >= 4 * nb * ms.I;
-        if (forced)
-          ok = ok && nb * ms.I <= maxv;
-        else
-          ok = ok && X->dims[tm] * 256 > (int64_t)device_info().l2 &&
-               (nb * ms.I * 64 <= nout || nout >= 8 * nb * ms.I);
-        if (ok) {
-          ms.tiled = true; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = q; t = tm;
-        }
-      }
+    } else {
+      int64_t Ioth[7];
+      for (int q = 0; q < N - 1; q++) Ioth[q] = X->dims[ms.other[q]];
+      decide_l2_block(ms, N, nout, ms.I, Ioth);
+      if (ms.tiled) t = ms.other[ms.tslot];
     }
     const int64_t nblk = ms.nblk;
     ms.Ivirt = ms.nblk * ms.I;

@@ -34,7 +34,8 @@ rep2 = B.cstf_factorize(X, [torch.from_numpy(f.copy()).cuda() for f in start], l
                         B.make_opts(R, outer_iters=outer, tol=tol, max_iter=10), comm=comm)   # back-to-back calls
 torch.cuda.synchronize()
 assert np.array_equal(rep["fit"], rep2["fit"]), (rep["fit"], rep2["fit"])
-out = {"fit": rep["fit"].tolist(), "iters": rep["iters"].tolist(), "comm_ms": rep["phase_ms"]["COMM"]}
+out = {"fit": rep["fit"].tolist(), "iters": rep["iters"].tolist(), "comm_ms": rep["phase_ms"]["COMM"],
+       "nblk": [X.layout(n)[0] for n in range(len(c.dims))]}
 if rank == 0:
     ref = oracle.coalesce(c.dims, idx, vals)
     orc = oracle.factorize(ref, start, outer_iters=outer, tol=tol, max_iter=10)
@@ -44,7 +45,7 @@ if rank == 0:
     out["fac_rel"] = max(float(np.max(np.abs(f.cpu().numpy() - g)) / np.max(np.abs(g)))
                          for f, g in zip(F, orc["factors"]))
     out["lam_rel"] = float(np.max(np.abs(lam.cpu().numpy() - orc["lam"][-1])) / np.max(np.abs(orc["lam"][-1])))
-print("RESULT", rank, json.dumps(out), flush=True)
+sys.stdout.write(f"RESULT {rank} " + json.dumps(out) + "\n"); sys.stdout.flush()   # one write: ranks share the pipe
 dist.destroy_process_group()
 '''
 
@@ -75,19 +76,25 @@ def run(tmp_path, nproc, case, port, comm="host"):
     (3, ("nell2", 40, 32, 0.0, 4), 29615, "0"),           # same case through the plain all-gather
     (1, ("nell2", 40, 32, 0.0, 4), 29616, "nccl"),        # a real NCCL communicator of one rank
     (1, ("enron", 60, 8, 1e-2, 5), 29617, "nccl"),
+    (2, ("nell2", 40, 32, 0.0, 4), 29618, "blk"),          # L2-blocked partitioned copies (forced)
+    (3, ("enron", 60, 16, 1e-2, 5), 29619, "blk"),
 ])
 def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port, peer, monkeypatch):
     """peer: CSTF_PEER_STORE for the host communicator, or "nccl" (one rank: the
     NCCL transport -- dlopen, unique id, init, all-reduce, all-gather -- and the
     partitioned layout with P = 1, the only NCCL job one GPU can run)."""
     comm = "nccl" if peer == "nccl" else "host"
-    monkeypatch.setenv("CSTF_PEER_STORE", "1" if peer == "nccl" else peer)
+    monkeypatch.setenv("CSTF_PEER_STORE", "1" if peer in ("nccl", "blk") else peer)
+    if peer == "blk":
+        monkeypatch.setenv("CSTF_L2_BLOCK_ROWS", "64")
     res = run(tmp_path, nproc, case, port, comm)
     r0 = res[0]
     for rk in range(1, nproc):          # every rank took the same decisions
         assert res[rk]["fit"] == r0["fit"] and res[rk]["iters"] == r0["iters"]
     assert r0["fit_rel"] <= 1e-6
-    if nproc > 1 and peer == "1" and case[3] == 0.0 and case[2] <= 32:
+    if peer == "blk":
+        assert all(max(res[rk]["nblk"]) > 1 for rk in range(nproc))     # some mode copy L2-blocked
+    if nproc > 1 and peer in ("1", "blk") and case[3] == 0.0 and case[2] <= 32:
         assert r0["comm_ms"] == 0.0          # no separate all-gather ran: rows were peer-stored
     if not r0["tie"]:
         assert r0["fac_rel"] <= 1e-6 and r0["lam_rel"] <= 1e-6

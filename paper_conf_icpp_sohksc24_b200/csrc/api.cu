@@ -586,7 +586,12 @@ cstf_status cstf_factorize_host(const cstf_tensor* X, const cstf_opts* opts, con
   HostIO io;
   io.in = dist ? nullptr : host_factors;
   io.out = host_factors;
-  CSTF_TRY(factorize_impl(X, opts, comm, d.data(), d_lam, report, st, &io));
+  const cstf_status fs = factorize_impl(X, opts, comm, d.data(), d_lam, report, st, &io);
+  if (fs != CSTF_OK) {               // no copy may touch the caller's buffers after the return
+    cudaStreamSynchronize(st);
+    cudaStreamSynchronize(w.copy);
+    return fs;
+  }
   if (host_lambda) CSTF_CUDA(cudaMemcpyAsync(host_lambda, d_lam, (size_t)R * 8, cudaMemcpyDeviceToHost, st));
   CSTF_CUDA(cudaStreamSynchronize(st));
   return CSTF_OK;

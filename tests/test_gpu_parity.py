@@ -583,6 +583,30 @@ def test_mttkrp_l2_blocked_long_rows_batches(B, R, monkeypatch):
     assert np.array_equal(host(M), first) and normwise(first, want) <= TOL
 
 
+@pytest.mark.parametrize("budget", [None, "1"])
+def test_mttkrp_l2_blocked_empty_blocks(B, budget, monkeypatch):
+    """Forced L2 blocks where most blocks of the blocked factor hold no nonzeros (and
+    rows of the output mode without nonzeros), whole-batch and one-block batches."""
+    monkeypatch.setenv("CSTF_L2_BLOCK_ROWS", "64")
+    if budget:
+        monkeypatch.setenv("CSTF_L2_BATCH_BYTES", budget)
+    dims = (50, 3000, 20)
+    idx, vals = datagen.coo(dims, (2, 2, 1), 40000, 41)
+    j = idx[1].astype(np.int64)
+    idx[1] = np.where(j < 1500, j % 500, 2500 + j % 500).astype(np.int32)   # blocks 8..38 empty
+    idx[0] = (idx[0] // 2 * 2).astype(np.int32)                              # odd rows empty
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    assert X.layout(0)[0] > 1
+    ref = oracle.coalesce(dims, idx, vals)
+    F = datagen.init_factors(dims, 16, 8)
+    Fd = [cu(f) for f in F]
+    M = cu(np.full((dims[0], 16), np.nan))
+    B.cstf_mttkrp(X, 0, Fd, M)
+    got = host(M)
+    assert normwise(got, oracle.mttkrp(ref, 0, F)) <= TOL
+    assert np.all(got[1::2] == 0.0)
+
+
 def test_factorize_bitwise_deterministic(B):
     """Fixed grids and fixed reduction orders everywhere: two runs are bit-identical."""
     c = datagen.CONFIGS["enron"].scaled(60, nnz_factor=1000)

@@ -36,7 +36,7 @@ bool rank_ok(int R) { return R >= 1 && R <= 128; }
 
 // Device-side scratch of one factorize / admm_update call, cached per device.
 struct DriverWs {
-  DevBuf grams, lam, inv, scal, flag, fitbuf, M, U, hostfac, Fi[8], S, stage;
+  DevBuf grams, lam, inv, scal, flag, fitbuf, fits, M, U, hostfac, Fi[8], S, stage;
   cudaStream_t copy = nullptr;   // host <-> device factor transfers of cstf_factorize_host
   cudaEvent_t ev_in[8] = {nullptr}, ev_out[8] = {nullptr};
   // distributed: all internal factor replicas in one allocation, mapped by the
@@ -232,6 +232,10 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   CSTF_TRY(w.scal.ensure((size_t)(8 + 2 * R) * 8));
   CSTF_TRY(w.flag.ensure(64));
   CSTF_TRY(w.fitbuf.ensure(300 * 8));
+  // with a fixed number of outer iterations (fit_tol = 0) the loop runs without a
+  // host round trip; the fits are collected at the end
+  const bool sync_each = o->fit_tol > 0.0;
+  if (!sync_each) CSTF_TRY(w.fits.ensure((size_t)2 * o->outer_iters * 8));
   CSTF_TRY(w.M.ensure((size_t)Imax * R * 8));
   CSTF_TRY(w.U.ensure((size_t)Usum * 8));
   double* G = w.grams.as<double>();
@@ -387,9 +391,14 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     // a8: fit of [[lambda^(N); H]]: inner product of M'(N) diag(mscale) with H_raw(N)
     tm.begin(N - 1, CSTF_PHASE_NORMALIZE);
     double* fb = w.fitbuf.as<double>();
+    double* fo = sync_each ? fb : w.fits.as<double>() + 2 * t;
     CSTF_TRY(fit(X->normX2, Iloc[N - 1], R, M, fac[N - 1] + off[N - 1], colscale, lam + (N - 1) * R, G, N, fb + 4,
-                 fb, flag, comm, st));
+                 fo, flag, comm, st));
     tm.end(N - 1, CSTF_PHASE_NORMALIZE);
+    if (!sync_each) {                 // fixed iteration count: no host round trip per iteration
+      if (rep) rep->outer_done = t + 1;
+      continue;
+    }
     CSTF_CUDA(cudaMemcpyAsync(w.host_small, fb, 8, cudaMemcpyDeviceToHost, st));
     CSTF_TRY(check_flag(flag, st));   // synchronises
     tm.collect();
@@ -398,8 +407,16 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       if (rep->fit) rep->fit[t] = f;
       rep->outer_done = t + 1;
     }
-    if (o->fit_tol > 0.0 && t > 0 && std::fabs(f - fit_prev) < o->fit_tol) break;
+    if (t > 0 && std::fabs(f - fit_prev) < o->fit_tol) break;
     fit_prev = f;
+  }
+  if (!sync_each) {                   // fits and the status flag of all iterations at once
+    std::vector<double> fits((size_t)2 * o->outer_iters);
+    CSTF_CUDA(cudaMemcpyAsync(fits.data(), w.fits.p, fits.size() * 8, cudaMemcpyDeviceToHost, st));
+    CSTF_TRY(check_flag(flag, st));   // synchronises
+    tm.collect();
+    if (rep && rep->fit)
+      for (int t = 0; t < o->outer_iters; t++) rep->fit[t] = fits[(size_t)2 * t];
   }
   // normalise the factors once (Alg. 1 l.11 applied to the final state)
   for (int n = 0; n < N; n++) {

@@ -370,9 +370,10 @@ def test_factorize_fixed_iterations_protocol(B):
         assert normwise(a, b) <= 1e-6
 
 
-@pytest.mark.parametrize("R,outer,tol,fit_tol,pinned", [(8, 3, 1e-2, 0.0, False), (32, 4, 0.0, 0.0, True),
-                                                       (16, 3, 0.0, 1e-12, True), (5, 1, 0.0, 0.0, False)])
-def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned):
+@pytest.mark.parametrize("R,outer,tol,fit_tol,pinned,update", [
+    (8, 3, 1e-2, 0.0, False, 0), (32, 4, 0.0, 0.0, True, 0), (16, 3, 0.0, 1e-12, True, 0),
+    (5, 1, 0.0, 0.0, False, 0), (16, 3, 0.0, 0.0, True, 1), (32, 2, 0.0, 0.0, True, 2)])
+def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned, update):
     """The host-buffer path (factor copies overlapped with the computation: factor 0
     copied in during MTTKRP(0), each final factor copied out after its last update)
     gives the bits of the device path."""
@@ -380,7 +381,7 @@ def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned):
     idx, vals = c.generate()
     X = B.cstf_tensor_load_coo(c.dims, idx, vals)
     start = datagen.init_factors(c.dims, R, 1)
-    opts = B.make_opts(R, outer_iters=outer, tol=tol, fit_tol=fit_tol)
+    opts = B.make_opts(R, outer_iters=outer, tol=tol, fit_tol=fit_tol, update=update)
     F = [cu(f) for f in start]
     lam = cu(np.zeros(R))
     g1 = B.cstf_factorize(X, F, lam, opts)

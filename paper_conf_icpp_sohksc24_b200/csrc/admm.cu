@@ -825,7 +825,9 @@ cstf_status launch_kernel(const KArgs& k, int& grid, bool gram, cudaStream_t st)
       case 40: return launch_dmma_t<40, false>(k, grid, st);
       case 48: return launch_dmma_t<48, false>(k, grid, st);
       case 56: return launch_dmma_t<56, false>(k, grid, st);
-      case 64: return launch_dmma_t<64, false>(k, grid, st);
+      case 64:
+        if (k.R == 64 && admm_pref()) return launch_dmma_t<64, false, false, false, true>(k, grid, st);
+        return launch_dmma_t<64, false>(k, grid, st);
     }
   }
   grid = (int)std::min<int64_t>(std::max<int64_t>(k.I, 1), (int64_t)device_info().sms * 8);

@@ -4,11 +4,19 @@ A step is one outer iteration of Alg. 1 over the whole
 tensor: for every mode S / rho / Cholesky / inverse, MTTKRP, the fused ADMM
 update (10 inner iterations, eps = 0: the paper's timing protocol L930-933),
 normalisation and Gram, then the fit.  Inputs are the seeded synthetic tensor
-of the chosen BASELINE.json config (default configs[1], NELL-2-shaped), already
-resident in HBM when the timed region starts.
+of the chosen BASELINE.json config, already resident in HBM when the timed
+region starts.  Default: configs[3], Delicious-4D-shaped -- the largest config
+the metric is quoted on at 1/2/4/8 B200 that fits one GPU (and the
+ADMM-update-bound one); configs[1] (nell2) and configs[2] (enron) are
+`--config` choices, configs[4] (amazon, 1.7B nonzeros) fits one GPU too but
+takes minutes to generate and load.
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--config nell2|enron|delicious|amazon]
-                  [--impl ours|reference] [--no-cpu-baseline]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config delicious|nell2|enron|amazon]
+                  [--impl ours|reference] [--no-cpu-baseline] [--comm nccl|host] [--ablation]
+
+--gpus N > 1 without torchrun re-launches itself under torch.distributed.run
+with N ranks (one per GPU over NCCL; --comm host lets the N ranks share one GPU
+to validate the multi-rank path).
 
 --impl reference times the FP64 CPU oracle (the reference arm of this tier) on
 the host cores: one outer iteration of the same workload per step.
@@ -49,11 +57,16 @@ def load_peaks():
 
 
 def measured_traffic(workload):
-    """DRAM bytes per launch of the dominant kernel from the committed ncu capture (or None)."""
+    """ncu DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) per launch of the
+    MTTKRP and ADMM kernels of every mode, from the committed capture
+    profiles/r02_traffic.json (or None)."""
     try:
-        with open(os.path.join(ROOT, "profiles", "r01_traffic.json")) as f:
-            t = json.load(f).get(workload)
-        return None if t is None else t["dram_read"] + t["dram_write"]
+        with open(os.path.join(ROOT, "profiles", "r02_traffic.json")) as f:
+            d = json.load(f)
+        t = d.get(workload)
+        if t is not None:
+            t = dict(t, source=d.get("source", "profiles/r02_traffic.json"))
+        return t
     except Exception:
         return None
 
@@ -146,35 +159,70 @@ def run_reference(args, cfg):
     return 0
 
 
-def admm_ablation(B, cfg, R, stream, reps=5):
-    """SURVEY f2 / Fig. 4 analogue on this workload's mode shapes: one ADMM update
-    (10 inner iterations, eps = 0) per mode, streaming vs row-resident kernel."""
+def admm_ablation(B, cfg, R, stream, reps=3):
+    """SURVEY f2 / Fig. 4 (Sec. 5.2) on this workload's mode shapes:
+    one ADMM update (10 passes, eps = 0) per mode for every arm -- the paper's
+    baseline (Alg. 2 as separate element-wise calls + two cuBLAS DTRSM per pass),
+    operation fusion only (OF), pre-inversion only (PI), both (OF+PI, the paper's
+    cuADMM shape), and libcstf's one-launch-per-pass (streaming) and row-resident
+    kernels.  S = Hadamard of the Grams (cstf_gram) of seeded normalised factors."""
     import torch
-    import oracle   # only to build a realistic S (Hadamard of Grams of normalised factors)
+    from paper_conf_icpp_sohksc24_b200 import ablation as AB
+    N = len(cfg.dims)
+    Gs = []
+    for k in range(N):
+        f = datagen.uniform(cfg.seed, 50 + k, 256 * R).reshape(256, R)
+        f = f / np.linalg.norm(f, axis=0)                       # column-normalised (reading D6)
+        g = torch.zeros(R, R, dtype=torch.float64, device="cuda")
+        B.cstf_gram(torch.from_numpy(f).cuda(), g)
+        Gs.append(g.cpu().numpy())
     out = {}
+
+    def timed(fn):
+        fn()                                                     # warm-up (also allocates workspaces)
+        ts = []
+        for _ in range(reps):
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            torch.cuda.synchronize()
+            a.record(stream)
+            fn()
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        return float(np.median(ts))
+
     for n, I in enumerate(cfg.dims):
-        Fs = [oracle.normalize(datagen.uniform(cfg.seed, 50 + k, 256 * R).reshape(256, R))[0]
-              for k in range(len(cfg.dims))]
-        S = torch.from_numpy(oracle.hadamard_except([oracle.gram(f) for f in Fs], n)).cuda()
+        S_h = np.ones((R, R))
+        for k in range(N):
+            if k != n:
+                S_h = S_h * Gs[k]
+        S = torch.from_numpy(S_h).cuda()
         M = torch.rand(I, R, dtype=torch.float64, device="cuda")
         H0 = torch.rand(I, R, dtype=torch.float64, device="cuda")
-        res = {}
+        H, U = H0.clone(), torch.zeros_like(H0)
+        res = {"rows": I}
+        for name, arm in (("baseline", AB.BASELINE), ("of", AB.OF), ("pi", AB.PI), ("of_pi", AB.OF_PI)):
+            res[name + "_ms"] = timed(lambda: AB.admm(arm, M, S, H, U, max_iter=10))
         for name, var in (("streaming", B.CSTF_ADMM_STREAMING), ("resident", B.CSTF_ADMM_RESIDENT)):
-            H, U = H0.clone(), torch.zeros_like(H0)
-            B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=var)
-            ts = []
-            for _ in range(reps):
-                a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                a.record(stream)
-                B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=var)
-                b.record(stream)
-                torch.cuda.synchronize()
-                ts.append(a.elapsed_time(b))
-            res[name + "_ms"] = float(np.median(ts))
-        res["speedup"] = res["streaming_ms"] / res["resident_ms"]
-        res["rows"] = I
+            res[name + "_ms"] = timed(lambda: B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=var))
+        for k in ("of", "pi", "of_pi", "streaming", "resident"):
+            res["speedup_" + k] = res["baseline_ms"] / res[k + "_ms"]
         out[f"mode{n}"] = res
+        del M, H0, H, U
+        torch.cuda.empty_cache()
     return out
+
+
+def relaunch_under_torchrun(n):
+    """--gpus N > 1 without a torchrun environment: run this command again as N ranks
+    (one process per GPU, rendezvous on 127.0.0.1)."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = sk.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    os.execv(sys.executable, cmd)
 
 
 def config_dict(cfg):
@@ -186,9 +234,9 @@ def config_dict(cfg):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=100)
+    ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="nell2", choices=sorted(datagen.CONFIGS))
+    ap.add_argument("--config", default="delicious", choices=sorted(datagen.CONFIGS))
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
@@ -203,12 +251,19 @@ def main():
     cfg = datagen.CONFIGS[args.config]
     if args.impl == "reference":
         return run_reference(args, cfg)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return relaunch_under_torchrun(args.gpus)
 
     import torch
     from paper_conf_icpp_sohksc24_b200 import binding as B
 
     rank, world, local = env_rank()
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: {world} ranks but --gpus {args.gpus}")
     host_comm = world > 1 and args.comm == "host"
+    if world > 1 and not host_comm and torch.cuda.device_count() < world:
+        raise SystemExit(f"bench.py: --gpus {world} over NCCL needs {world} GPUs, found "
+                         f"{torch.cuda.device_count()} (--comm host validates the multi-rank path on one GPU)")
     if host_comm:                            # validation: N ranks may share one GPU
         local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
@@ -271,53 +326,56 @@ def main():
     mp = rep["mode_phase_ms"]             # [N][5], summed over K steps
     ml = rep["mode_launches"]
     phase_ms = {k: v / K for k, v in rep["phase_ms"].items()}
-    # roofline of the dominant kernel
+    # roofline of the dominant kernel: algorithmic bytes / flops per launch
+    # over the CUDA-event time of that kernel's phase in the timed region
     peaks, peak_src = load_peaks()
     nnz = info["nnz"]
     mtt_ms = mp[:, 1].sum() / K
     upd_ms = mp[:, 2].sum() / K
-    admm_bytes_model = sum(10 * cm.admm_bytes(I, R) for I in cfg.dims)        # 40 I R per inner iteration
-    admm_gbs = admm_bytes_model / (upd_ms * 1e-3) / 1e9 if upd_ms > 0 else None
-    if mtt_ms >= upd_ms:
-        byts = sum(cm.mttkrp_bytes(nnz, cfg.dims, n, R) for n in range(N))
-        launches_per = N   # one MTTKRP per mode per step
-        ach = byts / (mtt_ms * 1e-3) / 1e9
-        roof = {"kernel": "mttkrp (k_mttkrp_fast + carry fix-up)", "bound": "hbm", "achieved": ach,
-                "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": ach / peaks["hbm_gbs"],
-                "traffic": measured_traffic(cfg.name), "traffic_source": "profiles/r01_traffic.json (ncu, mode 0)",
+    traffic = measured_traffic(cfg.name)          # ncu, one capture per kernel and mode (or None)
+    mtt_bytes = [cm.mttkrp_bytes(nnz, cfg.dims, n, R) for n in range(N)]
+    roof_mtt = {"kernel": "mttkrp (k_mttkrp_fast + carry fix-up)", "bound": "hbm",
+                "achieved": sum(mtt_bytes) / (mtt_ms * 1e-3) / 1e9, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "peak_source": peak_src,
-                "algorithmic_bytes_per_launch": byts / launches_per,
-                "avg_launch_ms": mtt_ms / launches_per,
-                "per_mode_ms": (mp[:, 1] / K).tolist()}
-        # second view (not the contract's roofline): factor-row bytes the kernel gathers
-        # (N-1 rows of R doubles per nonzero) vs the measured all-L1-hit gather ceiling
-        gathered = nnz * (N - 1) * R * 8 * N
-        line_gather = {"bound": "onchip_gather", "achieved": gathered / (mtt_ms * 1e-3) / 1e9,
-                       "peak": L1_GATHER_GBS, "unit": "GB/s",
-                       "frac": gathered / (mtt_ms * 1e-3) / 1e9 / L1_GATHER_GBS,
-                       "l2_gather_peak": L2_GATHER_GBS,
-                       "note": "factor-row bytes moved into registers (N-1 rows of R doubles per nonzero, "
-                               "L1 hits included) vs the all-L1-hit gather ceiling; meaningful when the "
-                               "factors are L2-resident",
-                       "peak_source": "tools/gather_probe.cu, profiles/r01_gather_probe.txt"}
-    else:
-        line_gather = None
-    # the ADMM update (the paper's cuADMM) against the FP64 datapath, always reported
-    fl_admm = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
-    roof_admm = {"kernel": "admm (k_admm_dmma, row-resident)", "bound": "fp64",
-                 "achieved": fl_admm / (upd_ms * 1e-3) / 1e12 if upd_ms > 0 else None,
+                "algorithmic_bytes_per_launch": sum(mtt_bytes) / N, "avg_launch_ms": mtt_ms / N,
+                "per_mode_ms": (mp[:, 1] / K).tolist(),
+                "traffic": None, "traffic_per_mode": None, "traffic_source": None}
+    roof_mtt["frac"] = roof_mtt["achieved"] / peaks["hbm_gbs"]
+    if traffic and "mttkrp" in traffic:
+        tm = traffic["mttkrp"]["per_mode_bytes"]
+        roof_mtt.update(traffic=sum(tm) / len(tm), traffic_per_mode=tm, traffic_source=traffic["source"],
+                        traffic_gbs=sum(tm) / (mtt_ms * 1e-3) / 1e9)
+    # the ADMM update (the paper's cuADMM, row-resident, FP64 tensor path): executed flops
+    # (DMMA products + the element-wise ops the FNN passes really run; not Eq. 3) against
+    # the measured FP64 peak, the ncu pipe fraction beside it
+    fl_exec = sum(cm.admm_flops_executed(I, R, 10, fnn=True, gram=R <= 32) for I in cfg.dims)
+    fl_eq3 = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
+    roof_admm = {"kernel": "admm (k_admm_dmma, row-resident, FNN passes)", "bound": "fp64",
+                 "achieved": fl_exec / (upd_ms * 1e-3) / 1e12 if upd_ms > 0 else None,
                  "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
-                 "frac": fl_admm / (upd_ms * 1e-3) / 1e12 / FP64_PEAK_TFLOPS if upd_ms > 0 else None,
-                 "note": "DMMA and DFMA share one FP64 datapath on B200 (profiles/r01_fp64_probe.txt); "
-                         "flops = (2R^2 + 19R) I per inner iteration (Eq. 3), 10 iterations per mode"}
-    if mtt_ms < upd_ms:
-        fl = fl_admm
-        ach = fl / (upd_ms * 1e-3) / 1e12
-        roof = {"kernel": "admm (k_admm_dmma, row-resident)", "bound": "tensor", "achieved": ach,
-                "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": ach / FP64_PEAK_TFLOPS,
-                "traffic": None, "peak_source": "measured FP64 DMMA peak (tools/microbench.cu, profiles/r01_microbench.txt)",
-                "algorithmic_flops_per_launch": fl / N, "avg_launch_ms": upd_ms / N,
-                "per_mode_ms": (mp[:, 2] / K).tolist()}
+                 "peak_source": "measured FP64 DMMA/DFMA peak: tools/microbench.cu -> profiles/r01_microbench.txt "
+                                "(MEASURED_PEAKS.json has no FP64 figure)",
+                 "flops": "executed: DMMA products 2 RP^2 + FNN element-wise 3R per pass + 13R last pass + "
+                          "fused Gram tiles, per row (costmodel.admm_flops_executed)",
+                 "eq3_flops_achieved": fl_eq3 / (upd_ms * 1e-3) / 1e12 if upd_ms > 0 else None,
+                 "per_mode_ms": (mp[:, 2] / K).tolist()}
+    roof_admm["frac"] = roof_admm["achieved"] / FP64_PEAK_TFLOPS if upd_ms > 0 else None
+    if traffic and "admm" in traffic:
+        ta = traffic["admm"]
+        roof_admm["ncu_fp64_datapath_frac"] = ta.get("fp64_datapath_frac")
+        roof_admm["ncu_source"] = traffic["source"]
+    # "ADMM update HBM GB/s" (BASELINE metric): measured DRAM bytes per ADMM launch (ncu)
+    # over the CUDA-event ADMM time; the paper's streaming byte model beside it, labelled
+    admm_gbs = {"model_40kIR_gbs": sum(10 * cm.admm_bytes(I, R) for I in cfg.dims) / (upd_ms * 1e-3) / 1e9
+                if upd_ms > 0 else None,
+                "model_note": "40 I R bytes per inner iteration (v1 streaming model), k = 10: NOT traffic",
+                "measured_gbs": None, "measured_bytes_per_step": None}
+    if traffic and "admm" in traffic and upd_ms > 0:
+        tb = sum(traffic["admm"]["per_mode_bytes"])
+        admm_gbs.update(measured_gbs=tb / (upd_ms * 1e-3) / 1e9, measured_bytes_per_step=tb,
+                        measured_source=traffic["source"],
+                        measured_frac_of_hbm=tb / (upd_ms * 1e-3) / 1e9 / peaks["hbm_gbs"])
+    roof = roof_mtt if mtt_ms >= upd_ms else dict(roof_admm, bound="fp64")
     line = {"metric": METRIC, "value": ms_step / 1e3, "unit": "s", "n_gpus": world, "steps": K,
             "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64",
@@ -326,7 +384,7 @@ def main():
                                                  "comm": "host callbacks (validation, shared GPU)" if host_comm
                                                  else "NCCL + CUDA-IPC peer stores"} if world > 1 else {})),
             "gpu_launches": int(launches),
-            "roofline": roof, "roofline_gather": line_gather, "roofline_admm": roof_admm, "admm_update_gbs": admm_gbs,
+            "roofline": roof, "roofline_admm": roof_admm, "admm_update_gbs": admm_gbs,
             "phases_ms_per_step": phase_ms, "clocks": clk,
             "setup": {"generate_s": t_gen, "load_coo_s": t_load, "nnz_coalesced": nnz}}
     # end to end through the public API with HOST buffers (pinned), one outer iteration per step

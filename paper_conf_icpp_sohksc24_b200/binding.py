@@ -75,12 +75,14 @@ _decl("cstf_status_string", ctypes.c_char_p, [c_int])
 _decl("cstf_last_error_message", ctypes.c_char_p, [])
 _decl("cstf_version", c_int, [])
 _decl("cstf_kernel_launch_count", c_int64, [])
+_decl("cstf_release_workspace", c_int, [])
 _decl("cstf_get_unique_id", c_int, [c_void_p])
 _decl("cstf_comm_create", c_int, [c_int, c_int, c_void_p, ctypes.POINTER(c_void_p)])
 _decl("cstf_comm_info", c_int, [c_void_p, ctypes.POINTER(c_int), ctypes.POINTER(c_int)])
 _ALLREDUCE_FN = ctypes.CFUNCTYPE(c_int, ctypes.POINTER(c_double), c_int64, c_void_p)
 _ALLGATHER_FN = ctypes.CFUNCTYPE(c_int, ctypes.POINTER(c_double), ctypes.POINTER(c_double), c_int64, c_void_p)
 _decl("cstf_comm_create_host", c_int, [c_int, c_int, _ALLREDUCE_FN, _ALLGATHER_FN, c_void_p, ctypes.POINTER(c_void_p)])
+_decl("cstf_comm_loopback", c_int, [c_int, c_void_p])
 _decl("cstf_comm_destroy", None, [c_void_p])
 _decl("cstf_partition_rows", c_int, [c_int64, c_void_p, c_int, c_void_p, c_void_p])
 _decl("cstf_tensor_load_coo", c_int, [c_int, c_void_p, c_int64, c_void_p, c_void_p, c_void_p, c_void_p,
@@ -104,12 +106,12 @@ _decl("cstf_factorize_host", c_int, [c_void_p, ctypes.POINTER(Opts), c_void_p, c
                                      ctypes.POINTER(Report), c_void_p])
 
 EXPORTED = ["cstf_status_string", "cstf_last_error_message", "cstf_version", "cstf_get_unique_id",
-            "cstf_comm_create", "cstf_comm_create_host", "cstf_comm_info", "cstf_comm_destroy",
+            "cstf_comm_create", "cstf_comm_create_host", "cstf_comm_loopback", "cstf_comm_info", "cstf_comm_destroy",
             "cstf_partition_rows",
             "cstf_tensor_load_coo", "cstf_tensor_info", "cstf_tensor_layout", "cstf_tensor_export_coo", "cstf_tensor_free",
             "cstf_mttkrp", "cstf_gram", "cstf_normalize", "cstf_admm_update", "cstf_hals_update",
             "cstf_mu_update", "cstf_factorize",
-            "cstf_factorize_host", "cstf_kernel_launch_count"]
+            "cstf_factorize_host", "cstf_kernel_launch_count", "cstf_release_workspace"]
 
 
 def _check(st, what):
@@ -149,6 +151,10 @@ def cstf_version() -> int:
 
 def cstf_kernel_launch_count() -> int:
     return _lib.cstf_kernel_launch_count()
+
+
+def cstf_release_workspace() -> None:
+    _check(_lib.cstf_release_workspace(), "cstf_release_workspace")
 
 
 def cstf_partition_rows(counts, nranks: int):
@@ -209,6 +215,14 @@ def cstf_comm_create_host(group=None) -> Comm:
     c = Comm(h.value)
     c._callbacks = cb          # keep the trampolines alive
     return c
+
+
+def cstf_comm_loopback(nparts: int) -> list:
+    """nparts communicators of one process (test backend: one thread per part, one
+    GPU); each thread passes its own handle to the library calls."""
+    arr = (c_void_p * nparts)()
+    _check(_lib.cstf_comm_loopback(int(nparts), arr), "cstf_comm_loopback")
+    return [Comm(arr[r]) for r in range(nparts)]
 
 
 def cstf_comm_create_nccl(group=None) -> Comm:

@@ -12,6 +12,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIBDIR = os.path.join(HERE, "lib")
 LIB = os.path.join(LIBDIR, "libcstf.so")
+ABL_SRC = os.path.join(HERE, "ablation", "ablation.cu")      # bench-only Fig. 4 arms (not part of libcstf)
+ABL_LIB = os.path.join(LIBDIR, "libcstf_ablation.so")
 ROOT = os.path.dirname(HERE)
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
@@ -45,7 +47,25 @@ def _stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
+def build_ablation(force: bool = False) -> str:
+    """libcstf_ablation.so: the paper's Fig. 4 ADMM arms (cuBLAS DGEAM/DTRSM/DGEMM + plain
+    kernels), used only by bench.py --ablation and tests/test_gpu_ablation.py."""
+    deps = [ABL_SRC, os.path.join(ROOT, "include", "cstf_ablation.h"), __file__]
+    if not force and os.path.exists(ABL_LIB) and all(os.path.getmtime(d) <= os.path.getmtime(ABL_LIB) for d in deps):
+        return ABL_LIB
+    os.makedirs(LIBDIR, exist_ok=True)
+    tmp = ABL_LIB + f".tmp{os.getpid()}"
+    cmd = [NVCC] + ARCH + ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2,-Wall", "-shared",
+                           "-o", tmp, ABL_SRC, "-lcublas"]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"nvcc failed for {ABL_SRC}:\n{r.stderr}")
+    os.replace(tmp, ABL_LIB)
+    return ABL_LIB
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
+    build_ablation(force)
     if not force and not _stale():
         return LIB
     os.makedirs(os.path.join(LIBDIR, "obj"), exist_ok=True)

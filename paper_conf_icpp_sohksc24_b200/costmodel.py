@@ -78,3 +78,28 @@ def gram_bytes(I: int, R: int) -> int:
 def gram_flops(I: int, R: int) -> int:
     """Upper triangle incl. diagonal, 2 flops per multiply-add."""
     return I * R * (R + 1)
+
+
+def admm_flops_executed(I: int, R: int, k: int, fnn: bool = True, gram: bool = True) -> int:
+    """FP64 flops the row-resident kernel (k_admm_dmma) actually executes for one
+    update of k passes with tol = 0, as opposed to Eq. 3:
+      * the R x R product on DMMA.8x8x4: 2 RP^2 per row and pass (RP = R rounded
+        up to a multiple of 8: padded columns are computed);
+      * element-wise, FNN passes (every pass but the last with the non-negativity
+        prox): x = H~ + w (DADD) and rho |x| + M (DFMA) = 3 flops per element
+        (the prox, |x| and the dual are sign-bit integer operations);
+      * the last pass (plain epilogue with the residual sums): A operand
+        (DADD + DFMA), x, H' - x, two residual differences, four DFMA sums
+        = 13 flops per element;
+      * the fused Gram epilogue: NT(NT+1)/2 tile pairs x 2 DMMA.8x8x4 per 8 rows.
+    Without FNN every pass costs the plain epilogue's A operand + x + dual = 5
+    flops per element, the last pass 13."""
+    RP = (R + 7) // 8 * 8
+    NT = RP // 8
+    prod = 2 * RP * RP * k
+    if fnn and k > 1:
+        elem = 3 * R * (k - 1) + 13 * R
+    else:
+        elem = 5 * R * max(k - 1, 0) + 13 * R
+    g = (NT * (NT + 1) // 2) * 2 * (8 * 8 * 4 * 2) / 8 if gram else 0
+    return int(I * (prod + elem + g))

@@ -884,6 +884,11 @@ bool gram_dmma(const double* d_H, int64_t I, int R, double* d_G, cudaStream_t st
 
 bool admm_can_fuse_gram(int R, double tol) { return tol == 0.0 && R <= 32; }
 
+void release_admm_ws() {
+  Workspace& w = ws();
+  for (DevBuf* b : {&w.slots, &w.sums, &w.out, &w.hs[0], &w.hs[1], &w.us[0], &w.us[1], &w.gpart}) b->release();
+}
+
 cstf_status hals_run(const UpdArgs& A, cudaStream_t st) {
   switch ((A.R + 7) & ~7) {
 #define C(RP) case RP: return launch_hals_t<RP>(A.M, A.H, A.S, A.mscale, A.hscale, A.I, A.R, A.sweeps, A.flag, st);

@@ -41,9 +41,11 @@ struct DriverWs {
   cudaEvent_t ev_in[8] = {nullptr}, ev_out[8] = {nullptr};
   // distributed: all internal factor replicas in one allocation, mapped by the
   // other ranks through CUDA IPC (NVLink peer memory) for the fused all-gather
-  DevBuf facall, xchg;
-  void* ipc_for = nullptr;
+  DevBuf facall, xchg, agreebuf;
+  uint64_t facall_gen = 0;       // bumped on every facall (re)allocation: equal on all ranks
+  uint64_t ipc_gen = ~0ull;      // facall_gen the peer mappings were made for
   const cstf_comm* ipc_comm = nullptr;
+  int ipc_state = 0;             // 0 none, 1 peers mapped, 2 agreed: no peer stores
   double* ipc_peer[8] = {nullptr};
   double* host_small = nullptr;  // pinned: fit, flags
   cudaStream_t side = nullptr;   // the R x R step of a mode overlaps its MTTKRP
@@ -68,31 +70,93 @@ DriverWs& dws() {
   return r;
 }
 
+// Agree on a status across ranks (a collective call returns the same
+// status on every rank).  Each rank contributes a one-hot vector of its status; the
+// all-reduced vector names every status that occurred, and all ranks return the
+// largest code.  A rank whose own call succeeded reports which status another rank hit.
+cstf_status agree(DriverWs& w, const cstf_comm* comm, cstf_status local, cudaStream_t st) {
+  if (comm_nranks(comm) <= 1) return local;
+  if (w.agreebuf.ensure(8 * 8) != CSTF_OK) return local;      // cannot agree: report the local status
+  double v[8] = {0};
+  v[(int)local & 7] = 1.0;
+  double* d = w.agreebuf.as<double>();
+  if (cudaMemcpyAsync(d, v, sizeof(v), cudaMemcpyHostToDevice, st) != cudaSuccess) return local;
+  if (comm_allreduce_f64(comm, d, 8, st) != CSTF_OK) return local;
+  if (cudaMemcpyAsync(v, d, sizeof(v), cudaMemcpyDeviceToHost, st) != cudaSuccess) return local;
+  if (cudaStreamSynchronize(st) != cudaSuccess) return local;
+  int worst = 0;
+  for (int k = 1; k < 8; k++)
+    if (v[k] > 0.0) worst = k;
+  if (worst == 0 || worst == (int)local) return local;
+  return fail((cstf_status)worst, std::string("another rank failed with ") + cstf_status_string((cstf_status)worst) +
+                                      (local != CSTF_OK ? std::string(" (this rank: ") + cstf_status_string(local) + ")"
+                                                        : std::string()));
+}
+
 // Map every other rank's factor replicas (CUDA IPC handles exchanged through the
-// communicator).  Collective; returns false on every rank if any rank fails.
+// communicator).  Collective on EVERY call: each rank says whether its mappings are
+// stale (facall re-allocated, other communicator, never decided); if any rank is
+// stale all ranks drop their mappings and redo the exchange, so no rank skips a
+// collective another rank enters, and no mapping outlives the allocation it was made
+// for.  Before opening a handle, the peer's device (PCI bus id) must be visible and
+// peer-accessible from ours (or be our own device).  Returns the same answer on every
+// rank: true only if every rank mapped every peer.
 bool open_peers(DriverWs& w, const cstf_comm* comm, cudaStream_t st) {
   const int P = comm_nranks(comm), me = comm_rank(comm);
-  if (w.ipc_for == w.facall.p && w.ipc_comm == comm) return true;
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+  constexpr int kW = 10;                       // doubles per rank: 64-byte handle + 16-byte PCI bus id
+  if (w.xchg.ensure((size_t)(kW * P + kW) * 8) != CSTF_OK) return false;
+  double* d = w.xchg.as<double>();
+  const bool stale = !(w.ipc_state != 0 && w.ipc_gen == w.facall_gen && w.ipc_comm == comm);
+  double flag = stale ? 1.0 : 0.0;
+  if (cudaMemcpyAsync(d, &flag, 8, cudaMemcpyHostToDevice, st) != cudaSuccess) return false;
+  if (comm_allreduce_f64(comm, d, 1, st) != CSTF_OK) return false;
+  if (cudaMemcpyAsync(&flag, d, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) return false;
+  if (cudaStreamSynchronize(st) != cudaSuccess) return false;
+  if (flag == 0.0) return w.ipc_state == 1;    // every rank fresh: the last (agreed) decision stands
   for (int r = 0; r < 8; r++)
     if (w.ipc_peer[r]) { cudaIpcCloseMemHandle(w.ipc_peer[r]); w.ipc_peer[r] = nullptr; }
-  w.ipc_for = nullptr;
+  w.ipc_state = 0;
   const char* env = getenv("CSTF_PEER_STORE");
   double ok = (P <= 8 && !(env && atoi(env) == 0)) ? 1.0 : 0.0;
-  cudaIpcMemHandle_t h;
-  memset(&h, 0, sizeof(h));
-  if (ok > 0 && cudaIpcGetMemHandle(&h, w.facall.p) != cudaSuccess) { cudaGetLastError(); ok = 0; }
-  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
-  if (w.xchg.ensure((size_t)(8 * P + 8) * 8) != CSTF_OK) return false;
-  double* d = w.xchg.as<double>();
-  if (cudaMemcpyAsync(d + 8 * P, &h, 64, cudaMemcpyHostToDevice, st) != cudaSuccess) return false;
-  if (comm_allgather_f64(comm, d + 8 * P, d, 8, st) != CSTF_OK) return false;
-  std::vector<cudaIpcMemHandle_t> hs((size_t)P);
-  if (cudaMemcpyAsync(hs.data(), d, (size_t)P * 64, cudaMemcpyDeviceToHost, st) != cudaSuccess) return false;
+  unsigned char mine[kW * 8];
+  memset(mine, 0, sizeof(mine));
+  int mydev = 0;
+  cudaGetDevice(&mydev);
+  if (ok > 0 && cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine), w.facall.p) != cudaSuccess) {
+    cudaGetLastError();
+    ok = 0;
+  }
+  if (cudaDeviceGetPCIBusId(reinterpret_cast<char*>(mine) + 64, 16, mydev) != cudaSuccess) {
+    cudaGetLastError();
+    ok = 0;
+  }
+  if (cudaMemcpyAsync(d + kW * P, mine, sizeof(mine), cudaMemcpyHostToDevice, st) != cudaSuccess) return false;
+  if (comm_allgather_f64(comm, d + kW * P, d, kW, st) != CSTF_OK) return false;
+  std::vector<unsigned char> all((size_t)P * kW * 8);
+  if (cudaMemcpyAsync(all.data(), d, all.size(), cudaMemcpyDeviceToHost, st) != cudaSuccess) return false;
   if (cudaStreamSynchronize(st) != cudaSuccess) return false;
   for (int r = 0; r < P && ok > 0; r++) {
     if (r == me) continue;
+    const unsigned char* rec = all.data() + (size_t)r * kW * 8;
+    char bus[17];
+    memcpy(bus, rec + 64, 16);
+    bus[16] = 0;
+    int pdev = -1, can = 0;
+    if (cudaDeviceGetByPCIBusId(&pdev, bus) != cudaSuccess) {      // peer GPU not visible here
+      cudaGetLastError();
+      ok = 0;
+      break;
+    }
+    if (pdev != mydev && (cudaDeviceCanAccessPeer(&can, mydev, pdev) != cudaSuccess || !can)) {
+      cudaGetLastError();
+      ok = 0;
+      break;
+    }
+    cudaIpcMemHandle_t h;
+    memcpy(&h, rec, 64);
     void* ptr = nullptr;
-    if (cudaIpcOpenMemHandle(&ptr, hs[(size_t)r], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
+    if (cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess) != cudaSuccess) {
       cudaGetLastError();
       ok = 0;
     } else {
@@ -105,13 +169,15 @@ bool open_peers(DriverWs& w, const cstf_comm* comm, cudaStream_t st) {
   if (comm_allreduce_f64(comm, d, 1, st) != CSTF_OK) return false;
   if (cudaMemcpyAsync(&fails, d, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess) return false;
   if (cudaStreamSynchronize(st) != cudaSuccess) return false;
+  w.ipc_gen = w.facall_gen;
+  w.ipc_comm = comm;
   if (fails > 0) {
     for (int r = 0; r < 8; r++)
       if (w.ipc_peer[r]) { cudaIpcCloseMemHandle(w.ipc_peer[r]); w.ipc_peer[r] = nullptr; }
+    w.ipc_state = 2;
     return false;
   }
-  w.ipc_for = w.facall.p;
-  w.ipc_comm = comm;
+  w.ipc_state = 1;
   return true;
 }
 
@@ -180,75 +246,93 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
                            cudaStream_t st, const HostIO* hio = nullptr) {
   const int N = X->N;
   const int R = o->R;
-  if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
-  if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
-  if (o->admm.prox < CSTF_PROX_NONNEG || o->admm.prox > CSTF_PROX_NONNEG_L1 || !(o->admm.alpha >= 0.0))
-    return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
-  if (o->update < CSTF_UPDATE_ADMM || o->update > CSTF_UPDATE_MU) return fail(CSTF_ERR_INVALID_ARG, "unknown update");
-  if (o->update == CSTF_UPDATE_MU && R > 64) return fail(CSTF_ERR_UNSUPPORTED, "MU update for R > 64");
   const bool dist = X->partitioned;
-  if ((comm != nullptr) != dist || comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
-    return fail(CSTF_ERR_INVALID_ARG, "comm does not match the tensor's partition");
-  for (int n = 0; n < N; n++)
-    if (!d_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");
   DriverWs& w = dws();
   // Distributed: every rank keeps full factors in the
   // internal (relabelled, zero-padded) row order; its own rows are the slice
   // [rank*B_n, (rank+1)*B_n).  Single GPU: the caller's buffers, all rows local.
-  std::vector<double*> fac(N);
+  std::vector<double*> fac(N), U(N);
   std::vector<int64_t> Ifull(N), Iloc(N), off(N), facoff(N);
-  if (dist) {                         // one allocation for all replicas (IPC-mappable)
-    int64_t tot = 0;
-    for (int n = 0; n < N; n++) {
-      facoff[n] = tot;
-      tot += ((int64_t)X->nranks * X->rows_per_rank[n] * R + 31) / 32 * 32;
-    }
-    CSTF_TRY(w.facall.ensure((size_t)tot * 8));
-  }
-  for (int n = 0; n < N; n++) {
-    if (dist) {
-      const int64_t B = X->rows_per_rank[n];
-      Ifull[n] = (int64_t)X->nranks * B;
-      Iloc[n] = B;
-      off[n] = (int64_t)X->rank * B * R;
-      fac[n] = w.facall.as<double>() + facoff[n];
-      CSTF_CUDA(cudaMemsetAsync(fac[n], 0, (size_t)Ifull[n] * R * 8, st));
-      CSTF_TRY(relabel_rows(d_factors[n], X->relabel[n].as<int32_t>(), X->dims[n], R, fac[n], 1, st));
-    } else {
-      Ifull[n] = Iloc[n] = X->dims[n];
-      off[n] = 0;
-      fac[n] = d_factors[n];
-    }
-  }
   int64_t Imax = 0, Usum = 0;
-  for (int n = 0; n < N; n++) { Imax = std::max(Imax, Iloc[n]); Usum += Iloc[n] * R; }
+  const bool sync_each = o->fit_tol > 0.0;
+  // Setup: validation and every allocation.  Distributed, its status is agreed over
+  // the ranks before the first collective of the algorithm, so a rank that fails
+  // here (bad argument, out of memory) makes every rank return the same status
+  // instead of leaving the others blocked in a collective.
+  auto setup = [&]() -> cstf_status {
+    if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
+    if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
+    if (o->admm.prox < CSTF_PROX_NONNEG || o->admm.prox > CSTF_PROX_NONNEG_L1 || !(o->admm.alpha >= 0.0))
+      return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
+    if (o->update < CSTF_UPDATE_ADMM || o->update > CSTF_UPDATE_MU) return fail(CSTF_ERR_INVALID_ARG, "unknown update");
+    if (o->update == CSTF_UPDATE_MU && R > 64) return fail(CSTF_ERR_UNSUPPORTED, "MU update for R > 64");
+    if ((comm != nullptr) != dist || comm_nranks(comm) != X->nranks || (dist && comm_rank(comm) != X->rank))
+      return fail(CSTF_ERR_INVALID_ARG, "comm does not match the tensor's partition");
+    for (int n = 0; n < N; n++)
+      if (!d_factors[n]) return fail(CSTF_ERR_INVALID_ARG, "factor pointer is NULL");
+    if (dist) {
+      const char* inj = getenv("CSTF_TEST_FAIL_RANK");     // tests: one rank fails its setup
+      if (inj && atoi(inj) == X->rank) return fail(CSTF_ERR_OUT_OF_MEMORY, "injected setup failure (CSTF_TEST_FAIL_RANK)");
+    }
+    if (dist) {                         // one allocation for all replicas (IPC-mappable)
+      int64_t tot = 0;
+      for (int n = 0; n < N; n++) {
+        facoff[n] = tot;
+        tot += ((int64_t)X->nranks * X->rows_per_rank[n] * R + 31) / 32 * 32;
+      }
+      const void* before = w.facall.p;
+      const size_t bytes_before = w.facall.bytes;
+      CSTF_TRY(w.facall.ensure((size_t)tot * 8));
+      // the size depends only on global sizes, so every rank re-allocates in the same call
+      if (w.facall.p != before || w.facall.bytes != bytes_before) w.facall_gen++;
+    }
+    for (int n = 0; n < N; n++) {
+      if (dist) {
+        const int64_t B = X->rows_per_rank[n];
+        Ifull[n] = (int64_t)X->nranks * B;
+        Iloc[n] = B;
+        off[n] = (int64_t)X->rank * B * R;
+        fac[n] = w.facall.as<double>() + facoff[n];
+        CSTF_CUDA(cudaMemsetAsync(fac[n], 0, (size_t)Ifull[n] * R * 8, st));
+        CSTF_TRY(relabel_rows(d_factors[n], X->relabel[n].as<int32_t>(), X->dims[n], R, fac[n], 1, st));
+      } else {
+        Ifull[n] = Iloc[n] = X->dims[n];
+        off[n] = 0;
+        fac[n] = d_factors[n];
+      }
+    }
+    for (int n = 0; n < N; n++) { Imax = std::max(Imax, Iloc[n]); Usum += Iloc[n] * R; }
+    CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
+    CSTF_TRY(w.lam.ensure((size_t)(N + 1) * R * 8));     // + R scratch for the initial column norms
+    CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
+    CSTF_TRY(w.S.ensure((size_t)R * R * 8));
+    CSTF_TRY(w.scal.ensure((size_t)(8 + 2 * R) * 8));
+    CSTF_TRY(w.flag.ensure(64));
+    CSTF_TRY(w.fitbuf.ensure(300 * 8));
+    // with a fixed number of outer iterations (fit_tol = 0) the loop runs without a
+    // host round trip; the fits are collected at the end
+    if (!sync_each) CSTF_TRY(w.fits.ensure((size_t)2 * o->outer_iters * 8));
+    CSTF_TRY(w.M.ensure((size_t)Imax * R * 8));
+    CSTF_TRY(w.U.ensure((size_t)Usum * 8));
+    int64_t uo = 0;
+    for (int n = 0; n < N; n++) { U[n] = w.U.as<double>() + uo; uo += Iloc[n] * R; }
+    CSTF_CUDA(cudaMemsetAsync(w.flag.p, 0, 4, st));
+    CSTF_CUDA(cudaMemsetAsync(w.U.p, 0, (size_t)Usum * 8, st));
+    return CSTF_OK;
+  };
+  {
+    cstf_status s0 = setup();
+    if (dist) s0 = agree(w, comm, s0, st);
+    if (s0 != CSTF_OK) return s0;
+  }
   // f4: fused all-gather through peer stores from the ADMM epilogue (falls back to
   // the NCCL / host all-gather when IPC mapping is unavailable or disabled)
   const bool peers = dist && open_peers(w, comm, st);
-  CSTF_TRY(w.grams.ensure((size_t)N * R * R * 8));
-  CSTF_TRY(w.lam.ensure((size_t)N * R * 8));
-  CSTF_TRY(w.inv.ensure((size_t)R * R * 8));
-  CSTF_TRY(w.S.ensure((size_t)R * R * 8));
-  CSTF_TRY(w.scal.ensure((size_t)(8 + 2 * R) * 8));
-  CSTF_TRY(w.flag.ensure(64));
-  CSTF_TRY(w.fitbuf.ensure(300 * 8));
-  // with a fixed number of outer iterations (fit_tol = 0) the loop runs without a
-  // host round trip; the fits are collected at the end
-  const bool sync_each = o->fit_tol > 0.0;
-  if (!sync_each) CSTF_TRY(w.fits.ensure((size_t)2 * o->outer_iters * 8));
-  CSTF_TRY(w.M.ensure((size_t)Imax * R * 8));
-  CSTF_TRY(w.U.ensure((size_t)Usum * 8));
   double* G = w.grams.as<double>();
   double* lam = w.lam.as<double>();
+  double* lam_scratch = lam + (size_t)N * R;
   double* M = w.M.as<double>();
   int* flag = w.flag.as<int>();
-  std::vector<double*> U(N);
-  {
-    int64_t off = 0;
-    for (int n = 0; n < N; n++) { U[n] = w.U.as<double>() + off; off += Iloc[n] * R; }
-  }
-  CSTF_CUDA(cudaMemsetAsync(flag, 0, 4, st));
-  CSTF_CUDA(cudaMemsetAsync(w.U.p, 0, (size_t)Usum * 8, st));
   const bool hin = hio && hio->in && !dist;
   const bool hout = hio && hio->out && !dist && o->fit_tol <= 0.0;
   if (hin) {                         // factors 1..N-1 first, factor 0 last (needed only by ADMM(0))
@@ -261,19 +345,22 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     }
   }
   // init (Alg. 1 l.1-5; readings D6): normalise, lambda = 1, G = H^T H
-  auto init_factor = [&](int n) -> cstf_status {
+  // (the column norms go to a scratch vector, never to lam: with host input, init of
+  // factor 0 runs after MTTKRP(0) while the side stream's Cholesky of mode 0 reads
+  // lam[0..R), which is set to 1 before the loop and not written again here)
+  auto init_factor = [&](int n, bool set_lam) -> cstf_status {
     double* Gn = G + (size_t)n * R * R;
     if (hin) CSTF_CUDA(cudaStreamWaitEvent(st, w.ev_in[n], 0));
     CSTF_TRY(gram_raw(fac[n], Ifull[n], R, Gn, st));
-    if (o->normalize_init) CSTF_TRY(normalize_from_gram(fac[n], Ifull[n], R, Gn, lam + n * R, st));
-    return fill(lam + n * R, R, 1.0, st);
+    if (o->normalize_init) CSTF_TRY(normalize_from_gram(fac[n], Ifull[n], R, Gn, lam_scratch, st));
+    return set_lam ? fill(lam + n * R, R, 1.0, st) : CSTF_OK;
   };
   for (int n = 0; n < N; n++) {      // factors are replicated: redundant, no communication
     if (hin && n == 0) {             // deferred: after MTTKRP(0) is queued
       CSTF_TRY(fill(lam, R, 1.0, st));
       continue;
     }
-    CSTF_TRY(init_factor(n));
+    CSTF_TRY(init_factor(n, true));
   }
   if (peers) {   // no rank may peer-store into a replica another rank is still initialising / reading
     CSTF_TRY(comm_allreduce_f64(comm, w.xchg.as<double>(), 1, st));
@@ -320,7 +407,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       // a2: MTTKRP of the raw factors (MTTKRP phase = both, overlapped)
       tm.begin(n, CSTF_PHASE_MTTKRP);
       CSTF_TRY(mttkrp(X, n, R, fac.data(), M, st, nullptr));
-      if (hin && t == 0 && n == 0) CSTF_TRY(init_factor(0));   // its copy overlapped MTTKRP(0)
+      if (hin && t == 0 && n == 0) CSTF_TRY(init_factor(0, false));   // its copy overlapped MTTKRP(0)
       CSTF_CUDA(cudaStreamWaitEvent(st, w.join, 0));
       tm.end(n, CSTF_PHASE_MTTKRP);
       // a5: ADMM on M diag(mscale); warm start H_raw (D4) or the normalised H (literal)
@@ -400,7 +487,11 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       continue;
     }
     CSTF_CUDA(cudaMemcpyAsync(w.host_small, fb, 8, cudaMemcpyDeviceToHost, st));
-    CSTF_TRY(check_flag(flag, st));   // synchronises
+    {                                 // synchronises; the flags derive from replicated / all-reduced
+      cstf_status fs = check_flag(flag, st);     // values, the agreement makes that explicit
+      if (dist) fs = agree(w, comm, fs, st);
+      CSTF_TRY(fs);
+    }
     tm.collect();
     const double f = w.host_small[0];
     if (rep) {
@@ -413,7 +504,11 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   if (!sync_each) {                   // fits and the status flag of all iterations at once
     std::vector<double> fits((size_t)2 * o->outer_iters);
     CSTF_CUDA(cudaMemcpyAsync(fits.data(), w.fits.p, fits.size() * 8, cudaMemcpyDeviceToHost, st));
-    CSTF_TRY(check_flag(flag, st));   // synchronises
+    {
+      cstf_status fs = check_flag(flag, st);     // synchronises
+      if (dist) fs = agree(w, comm, fs, st);
+      CSTF_TRY(fs);
+    }
     tm.collect();
     if (rep && rep->fit)
       for (int t = 0; t < o->outer_iters; t++) rep->fit[t] = fits[(size_t)2 * t];
@@ -570,6 +665,23 @@ cstf_status cstf_hals_update(const double* d_M, const double* d_S, double* d_H, 
 cstf_status cstf_mu_update(const double* d_M, const double* d_S, double* d_H, int64_t I, int R, int sweeps,
                            void* stream) {
   return run_update(CSTF_UPDATE_MU, d_M, d_S, d_H, I, R, sweeps, stream);
+}
+
+cstf_status cstf_release_workspace(void) {
+  CSTF_CUDA(cudaDeviceSynchronize());       // no launch of this thread may still use them
+  DriverWs& w = dws();
+  for (int r = 0; r < 8; r++)
+    if (w.ipc_peer[r]) { cudaIpcCloseMemHandle(w.ipc_peer[r]); w.ipc_peer[r] = nullptr; }
+  w.ipc_state = 0;
+  for (DevBuf* b : {&w.grams, &w.lam, &w.inv, &w.scal, &w.flag, &w.fitbuf, &w.fits, &w.M, &w.U, &w.hostfac, &w.S,
+                    &w.stage, &w.facall, &w.xchg, &w.agreebuf})
+    b->release();
+  for (int n = 0; n < 8; n++) w.Fi[n].release();
+  w.facall_gen++;
+  release_mttkrp_ws();
+  release_admm_ws();
+  release_dense_ws();
+  return CSTF_OK;
 }
 
 cstf_status cstf_factorize(const cstf_tensor* X, const cstf_opts* opts, const cstf_comm* comm,

@@ -349,6 +349,12 @@ Workspace& ws() {
 
 }  // namespace
 
+void release_dense_ws() {
+  Workspace& w = ws();
+  w.part.release();
+  w.linv.release();
+}
+
 cstf_status fill(double* d, int64_t n, double v, cudaStream_t st) {
   if (n <= 0) return CSTF_OK;
   int g = (int)std::min<int64_t>((n + 255) / 256, (int64_t)device_info().sms * 16);

@@ -69,6 +69,7 @@ struct Comm {
   cstf_host_allreduce_fn host_allreduce = nullptr;   // host-callback transport
   cstf_host_allgather_fn host_allgather = nullptr;
   void* user = nullptr;
+  void* loop = nullptr;  // cstf_comm_loopback member (owned)
 };
 cstf_status comm_allreduce_f64(const cstf_comm* c, double* d_buf, size_t count, cudaStream_t st);
 cstf_status comm_allgather_f64(const cstf_comm* c, const double* d_send, double* d_recv,
@@ -224,6 +225,11 @@ struct UpdArgs {
   int sweeps;
 };
 cstf_status hals_run(const UpdArgs& a, cudaStream_t st);
+
+// cached per-thread, per-device workspaces (cstf_release_workspace)
+void release_mttkrp_ws();
+void release_admm_ws();
+void release_dense_ws();
 cstf_status mu_run(const UpdArgs& a, cudaStream_t st);
 
 }  // namespace cstf

@@ -531,9 +531,12 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
   if (const char* be = getenv("CSTF_L2_BATCH_BYTES")) {
     budget = (size_t)atoll(be);
   } else {
+    // at most a quarter of the device and half of what is free (counting the buffer
+    // already cached); the summation order does not depend on the batch size (each
+    // batch continues M's running sum in block order), so neither do the results
     size_t fr = 0, tot = 0;
     CSTF_CUDA(cudaMemGetInfo(&fr, &tot));
-    budget = tot / 4;
+    budget = std::min(tot / 4, (fr + w.partial.bytes) / 2);
   }
   int64_t B = std::max<int64_t>(1, std::min<int64_t>(nblk, (int64_t)(budget / std::max<size_t>(per_block, 1))));
   while (w.partial.ensure((size_t)B * per_block) != CSTF_OK) {
@@ -558,18 +561,33 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
   // CSTF_L2_PERSIST=<bytes> overrides (0 disables).
   size_t persist = (nnz / std::max<int64_t>(nblk, 1) >= ((int64_t)16 << 20)) ? ((size_t)64 << 20) : 0;
   if (const char* pe = getenv("CSTF_L2_PERSIST")) persist = (size_t)atoll(pe);
+  // The caller's persisting-L2 limit and the stream's access-policy window are saved
+  // here and restored after the blocked launches (no process-wide state
+  // left changed by a stream-ordered library call).
+  size_t saved_limit = 0;
+  cudaStreamAttrValue saved_win = {};
+  bool restore_limit = false, restore_win = false;
   if (persist) {
     int maxp = 0;
     cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, di.device);
     persist = std::min<size_t>(persist, (size_t)std::max(maxp, 0));
-    static thread_local size_t set_for[64] = {0};
-    if (persist && set_for[di.device & 63] != persist) {
+    if (persist && cudaDeviceGetLimit(&saved_limit, cudaLimitPersistingL2CacheSize) != cudaSuccess) {
+      cudaGetLastError();
+      persist = 0;
+    }
+    if (persist && saved_limit != persist) {
       if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, persist) == cudaSuccess) {
-        set_for[di.device & 63] = persist;
+        restore_limit = true;
       } else {                    // not available (e.g. MIG): plain launches, no error
         cudaGetLastError();
         persist = 0;
       }
+    }
+    if (persist) {
+      if (cudaStreamGetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &saved_win) == cudaSuccess)
+        restore_win = true;
+      else
+        cudaGetLastError();
     }
   }
   for (int64_t b0 = 0; b0 < nblk; b0 += B) {
@@ -639,18 +657,27 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     (*nl)++;
   }
   if (persist) {
-    // drop the window; once the launches have run, release the persisting lines (the
-    // reset is not stream-ordered) so later kernels get the whole L2 back
+    // restore the caller's window; once the launches have run, release the persisting
+    // lines (cudaCtxResetPersistingL2Cache is not stream-ordered, hence the one host
+    // synchronisation of this path) and restore the caller's set-aside
     cudaStreamAttrValue v = {};
-    v.accessPolicyWindow.num_bytes = 0;
+    if (restore_win) v = saved_win;
+    else v.accessPolicyWindow.num_bytes = 0;
     if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v) != cudaSuccess) cudaGetLastError();
     CSTF_CUDA(cudaStreamSynchronize(st));
     if (cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
+    if (restore_limit && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, saved_limit) != cudaSuccess)
+      cudaGetLastError();
   }
   return CSTF_OK;
 }
 
 }  // namespace
+
+void release_mttkrp_ws() {
+  Workspace& w = ws();
+  for (DevBuf* b : {&w.lb, &w.cont, &w.carry, &w.gsum, &w.partial, &w.kbptr, &w.queue}) b->release();
+}
 
 cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d_factors,
                    double* d_M, cudaStream_t st, int64_t* launches) {

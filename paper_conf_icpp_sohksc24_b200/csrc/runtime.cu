@@ -5,6 +5,8 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
+#include <condition_variable>
 #include <cstring>
 #include <mutex>
 #include <numeric>
@@ -214,6 +216,92 @@ cstf_status cstf_comm_create_host(int nranks, int rank, cstf_host_allreduce_fn a
   return CSTF_OK;
 }
 
+}  // extern "C"
+
+// ------------------------------------------------------------------ loopback group
+// cstf_comm_loopback: nparts communicators of ONE process (one thread per part,
+// sharing a GPU).  Collectives meet at a host barrier; the all-reduce sums the
+// parts' host copies in rank order (identical bits on every part), the all-gather
+// concatenates them.  A part that does not arrive within kLoopTimeout makes the
+// collective fail (CSTF_ERR_NCCL) instead of hanging.
+namespace {
+constexpr auto kLoopTimeout = std::chrono::seconds(120);
+struct LoopGroup {
+  int n = 0;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t gen = 0;
+  bool broken = false;
+  std::vector<const double*> src;
+  std::atomic<int> refs{0};
+  bool barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    if (broken) return false;
+    const uint64_t g = gen;
+    if (++arrived == n) {
+      arrived = 0;
+      gen++;
+      cv.notify_all();
+      return true;
+    }
+    if (!cv.wait_for(lk, kLoopTimeout, [&] { return gen != g || broken; }) || broken) {
+      broken = true;
+      cv.notify_all();
+      return false;
+    }
+    return true;
+  }
+};
+struct LoopMember {
+  LoopGroup* g;
+  int rank;
+};
+int loop_allreduce(double* buf, int64_t count, void* user) {
+  LoopMember* m = static_cast<LoopMember*>(user);
+  LoopGroup* g = m->g;
+  std::vector<double> mine(buf, buf + count);
+  g->src[(size_t)m->rank] = mine.data();
+  if (!g->barrier()) return 1;
+  for (int64_t i = 0; i < count; i++) {
+    double s = 0.0;
+    for (int r = 0; r < g->n; r++) s += g->src[(size_t)r][i];
+    buf[i] = s;
+  }
+  return g->barrier() ? 0 : 1;       // nobody releases `mine` while others still read it
+}
+int loop_allgather(const double* send, double* recv, int64_t count, void* user) {
+  LoopMember* m = static_cast<LoopMember*>(user);
+  LoopGroup* g = m->g;
+  g->src[(size_t)m->rank] = send;
+  if (!g->barrier()) return 1;
+  for (int r = 0; r < g->n; r++) memcpy(recv + (size_t)r * count, g->src[(size_t)r], (size_t)count * 8);
+  return g->barrier() ? 0 : 1;
+}
+}  // namespace
+
+extern "C" {
+
+cstf_status cstf_comm_loopback(int nparts, cstf_comm** out) {
+  if (!out || nparts < 1 || nparts > 64) return fail(CSTF_ERR_INVALID_ARG, "cstf_comm_loopback arguments");
+  LoopGroup* g = new LoopGroup();
+  g->n = nparts;
+  g->src.assign((size_t)nparts, nullptr);
+  g->refs = nparts;
+  for (int r = 0; r < nparts; r++) {
+    cstf_comm* c = new cstf_comm();
+    c->c.nranks = nparts;
+    c->c.rank = r;
+    c->c.host_allreduce = loop_allreduce;
+    c->c.host_allgather = loop_allgather;
+    LoopMember* m = new LoopMember{g, r};
+    c->c.user = m;
+    c->c.loop = m;
+    out[r] = c;
+  }
+  return CSTF_OK;
+}
+
 cstf_status cstf_comm_info(const cstf_comm* comm, int* nranks, int* rank) {
   if (!comm) return fail(CSTF_ERR_INVALID_ARG, "comm is NULL");
   if (nranks) *nranks = comm->c.nranks;
@@ -224,6 +312,11 @@ cstf_status cstf_comm_info(const cstf_comm* comm, int* nranks, int* rank) {
 void cstf_comm_destroy(cstf_comm* comm) {
   if (!comm) return;
   if (comm->c.nccl && g_nccl.CommDestroy) g_nccl.CommDestroy((ncclComm_t)comm->c.nccl);
+  if (comm->c.loop) {
+    LoopMember* m = static_cast<LoopMember*>(comm->c.loop);
+    if (--m->g->refs == 0) delete m->g;
+    delete m;
+  }
   delete comm;
 }
 

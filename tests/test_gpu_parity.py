@@ -370,10 +370,11 @@ def test_factorize_fixed_iterations_protocol(B):
         assert normwise(a, b) <= 1e-6
 
 
-@pytest.mark.parametrize("R,outer,tol,fit_tol,pinned,update", [
-    (8, 3, 1e-2, 0.0, False, 0), (32, 4, 0.0, 0.0, True, 0), (16, 3, 0.0, 1e-12, True, 0),
-    (5, 1, 0.0, 0.0, False, 0), (16, 3, 0.0, 0.0, True, 1), (32, 2, 0.0, 0.0, True, 2)])
-def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned, update):
+@pytest.mark.parametrize("R,outer,tol,fit_tol,pinned,update,warm", [
+    (8, 3, 1e-2, 0.0, False, 0, 0), (32, 4, 0.0, 0.0, True, 0, 0), (16, 3, 0.0, 1e-12, True, 0, 0),
+    (5, 1, 0.0, 0.0, False, 0, 0), (16, 3, 0.0, 0.0, True, 1, 0), (32, 2, 0.0, 0.0, True, 2, 0),
+    (32, 3, 0.0, 0.0, True, 0, 1), (8, 3, 1e-2, 0.0, False, 0, 1)])
+def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned, update, warm):
     """The host-buffer path (factor copies overlapped with the computation: factor 0
     copied in during MTTKRP(0), each final factor copied out after its last update)
     gives the bits of the device path."""
@@ -381,7 +382,7 @@ def test_factorize_host_matches_device(B, R, outer, tol, fit_tol, pinned, update
     idx, vals = c.generate()
     X = B.cstf_tensor_load_coo(c.dims, idx, vals)
     start = datagen.init_factors(c.dims, R, 1)
-    opts = B.make_opts(R, outer_iters=outer, tol=tol, fit_tol=fit_tol, update=update)
+    opts = B.make_opts(R, outer_iters=outer, tol=tol, fit_tol=fit_tol, update=update, warm=warm)
     F = [cu(f) for f in start]
     lam = cu(np.zeros(R))
     g1 = B.cstf_factorize(X, F, lam, opts)
@@ -547,7 +548,7 @@ def test_mttkrp_l2_blocked_default(B, monkeypatch):
         assert normwise(first, host(Mp)) <= TOL, n
 
 
-@pytest.mark.parametrize("R", [16, 32])
+@pytest.mark.parametrize("R", [16, 32, 64])
 def test_mttkrp_l2_blocked_long_rows_batches(B, R, monkeypatch):
     """Default L2 blocking of a long-row output mode (the Amazon case: >= 8 nonzeros per
     (row, block)); blocks processed in batches of any size (forced small budgets)

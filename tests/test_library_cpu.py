@@ -126,3 +126,30 @@ dist.destroy_process_group()
                          env=env, capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr[-3000:]
     assert out.stdout.count("OK") == 2, out.stdout + out.stderr[-2000:]
+
+
+def test_loopback_comms_without_gpu(lib):
+    """cstf_comm_loopback (SURVEY s8(b) test backend): nparts handles with ranks
+    0..nparts-1 of one group, created and destroyed without a device."""
+    comms = lib.cstf_comm_loopback(3)
+    assert [c.info() for c in comms] == [(3, 0), (3, 1), (3, 2)]
+    del comms
+    arr = (ctypes.c_void_p * 1)()
+    assert lib._lib.cstf_comm_loopback(0, arr) == lib.CSTF_ERR_INVALID_ARG
+    assert lib._lib.cstf_comm_loopback(65, arr) == lib.CSTF_ERR_INVALID_ARG
+
+
+def test_ablation_library_exports():
+    """The bench-only Fig. 4 library (include/cstf_ablation.h) builds and exports its ABI."""
+    from paper_conf_icpp_sohksc24_b200 import build
+    path = build.build_ablation()
+    so = ctypes.CDLL(path)
+    txt = re.sub(r"/\*.*?\*/", "", open(os.path.join(ROOT, "include", "cstf_ablation.h")).read(), flags=re.S)
+    syms = set(re.findall(r"\b(cstf_[a-z_0-9]+)\s*\(", txt))
+    assert syms == {"cstf_ablation_admm", "cstf_ablation_last_error", "cstf_ablation_last_calls"}
+    for s in syms:
+        assert hasattr(so, s)
+    so.cstf_ablation_admm.restype = ctypes.c_int
+    so.cstf_ablation_last_error.restype = ctypes.c_char_p
+    rc = so.cstf_ablation_admm(7, None, None, None, None, ctypes.c_int64(10), 8, 10, None, None)
+    assert rc != 0 and b"arm" in so.cstf_ablation_last_error()

@@ -502,3 +502,90 @@ def test_f1_factorize_schemes_on_planted(rng):
         r = oracle.factorize(X, start, outer_iters=30, max_iter=1, update=upd)
         assert r["fit"][-1] > 0.99
         assert np.all(np.diff(r["fit"]) > -1e-9)
+
+
+# --------------------------------------------------------------------- D11 outer stopping rule
+def test_D11_fit_tol_stops_at_first_small_change(rng):
+    """D11 (L505 "until convergence"): with fit_tol > 0 the outer loop stops after the
+    first outer iteration t >= 1 whose fit changed by less than fit_tol.  The stop index
+    is read off a fixed-count run of the same problem (the loop is deterministic), and
+    the early-stopped run must reproduce that run's prefix bit for bit."""
+    dims = (30, 25, 20)
+    idx, vals = random_coo(rng, dims, 1500, dup_frac=0.0, neg=False, zeros=False)
+    X = oracle.coalesce(dims, idx, vals)
+    start = [rng.random((I, 4)) for I in dims]
+    T = 8
+    full = oracle.factorize(X, start, outer_iters=T, tol=0.0, max_iter=5)
+    f = full["fit"]
+    assert len(f) == T
+    d = np.abs(np.diff(f))                                 # d[t-1] = |fit_t - fit_{t-1}|
+    # the first t >= 2 whose change is a new minimum, and a tolerance strictly between
+    tstar = next(t for t in range(2, T) if d[t - 1] < np.min(d[:t - 1]))
+    tol = np.sqrt(d[tstar - 1] * np.min(d[:tstar - 1]))
+    assert d[tstar - 1] < tol < np.min(d[:tstar - 1])
+    early = oracle.factorize(X, start, outer_iters=T, tol=0.0, max_iter=5, fit_tol=tol)
+    assert len(early["fit"]) == tstar + 1
+    assert np.array_equal(early["fit"], f[:tstar + 1])
+    ref = oracle.factorize(X, start, outer_iters=tstar + 1, tol=0.0, max_iter=5)
+    for a, b in zip(early["factors"], ref["factors"]):
+        assert np.array_equal(a, b)
+    # a tolerance below every change never stops early; fit_tol = 0 disables the test
+    never = oracle.factorize(X, start, outer_iters=T, tol=0.0, max_iter=5, fit_tol=0.5 * np.min(d))
+    assert len(never["fit"]) == T
+
+
+# --------------------------------------------------------------------- D6 normalize_init = 0
+def test_D6_unnormalised_start_reaches_the_same_scale_free_update(rng):
+    """normalize_init = 0 (the caller's factors used as given, lambda = 1).  The
+    converged ADMM update of mode n is the per-row NNLS solution of (M, S) (P2), which
+    is scale covariant: with every other factor scaled by a positive diagonal D_k,
+    M -> M D and S -> D S D (D = prod D_k), so the NNLS solution is H D^{-1} and its
+    column normalisation is unchanged.  One outer iteration with converged updates
+    therefore gives the same normalised factors, lambda and fit from raw scaled factors
+    (normalize_init = 0) as from the normalised ones (normalize_init = 1).  A dropped or
+    misplaced scale anywhere in the branch (Grams, MTTKRP or warm start of raw factors)
+    breaks the equality."""
+    dims = (14, 11, 9)
+    idx, vals = random_coo(rng, dims, 600, dup_frac=0.0, neg=False, zeros=False)
+    X = oracle.coalesce(dims, idx, vals)
+    R = 3
+    base = [oracle.normalize(rng.random((I, R)) + 0.05)[0] for I in dims]
+    raw = [b * (0.3 + 4.0 * rng.random(R)) for b in base]           # columns scaled by D_k
+    a = oracle.factorize(X, base, outer_iters=1, tol=0.0, max_iter=6000, normalize_init=True)
+    b = oracle.factorize(X, raw, outer_iters=1, tol=0.0, max_iter=6000, normalize_init=False)
+    for fa, fb in zip(a["factors"], b["factors"]):
+        assert normwise(fb, fa) <= 1e-9
+    assert normwise(b["lam"][-1], a["lam"][-1]) <= 1e-9
+    assert abs(b["fit"][0] - a["fit"][0]) <= 1e-9
+    # with few passes the warm start differs (raw vs normalised H), so the branches differ
+    a10 = oracle.factorize(X, base, outer_iters=1, tol=0.0, max_iter=3, normalize_init=True)
+    b10 = oracle.factorize(X, raw, outer_iters=1, tol=0.0, max_iter=3, normalize_init=False)
+    assert normwise(b10["factors"][0], a10["factors"][0]) > 1e-6
+    # normalize_init = 0 on already normalised factors is the normalize_init = 1 run on them
+    c = oracle.factorize(X, base, outer_iters=2, tol=1e-2, max_iter=10, normalize_init=False)
+    d = oracle.factorize(X, [oracle.normalize(f)[0] for f in base], outer_iters=2, tol=1e-2, max_iter=10,
+                         normalize_init=True)
+    for fc, fd in zip(c["factors"], d["factors"]):
+        assert normwise(fc, fd) <= 1e-12
+
+
+def test_D6_initial_lambda_is_one_in_both_branches(rng):
+    """Reading D6: the initial lambda is exactly 1 whether or not the factors are
+    normalised first, so the scaled (D4) and literal warm starts coincide for the
+    first update of every mode; after one outer iteration the factors (each mode's
+    first update, normalised) must be bit-identical across the two warm-start
+    readings, and after two (lambda = the previous column norms) they differ."""
+    dims = (12, 10, 9)
+    idx, vals = random_coo(rng, dims, 500, dup_frac=0.0, neg=False, zeros=False)
+    X = oracle.coalesce(dims, idx, vals)
+    raw = [rng.random((I, 4)) * 3.0 for I in dims]
+    for ni in (False, True):
+        w0 = oracle.factorize(X, raw, outer_iters=1, tol=0.0, max_iter=4, normalize_init=ni, warm=oracle.WARM_SCALED)
+        w1 = oracle.factorize(X, raw, outer_iters=1, tol=0.0, max_iter=4, normalize_init=ni,
+                              warm=oracle.WARM_NORMALIZED)
+        for a, b in zip(w0["factors"], w1["factors"]):
+            assert np.array_equal(a, b), ni
+        v0 = oracle.factorize(X, raw, outer_iters=2, tol=0.0, max_iter=4, normalize_init=ni, warm=oracle.WARM_SCALED)
+        v1 = oracle.factorize(X, raw, outer_iters=2, tol=0.0, max_iter=4, normalize_init=ni,
+                              warm=oracle.WARM_NORMALIZED)
+        assert normwise(v0["factors"][0], v1["factors"][0]) > 1e-6

@@ -100,16 +100,33 @@ __global__ void k_chol(const double* __restrict__ S, int R, int want_inv, double
   }
 }
 
+// Element-wise kernels: 16-byte (double2) accesses over the flat I x R array, grid
+// = 16 CTAs per SM (enough 16-byte loads in flight to stream at HBM rate); an odd
+// element count leaves one scalar tail element for thread 0 of CTA 0.
+template <class F2, class F1>
+__device__ __forceinline__ void elemwise(int64_t n, F2 body2, F1 body1) {
+  const int64_t n2 = n >> 1;
+  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n2; x += (int64_t)gridDim.x * kT) body2(x);
+  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) body1(n - 1);
+}
+__device__ __forceinline__ double2 ld2(const double* p, int64_t x) { return reinterpret_cast<const double2*>(p)[x]; }
+__device__ __forceinline__ void st2(double* p, int64_t x, double a, double b) {
+  reinterpret_cast<double2*>(p)[x] = make_double2(a, b);
+}
+__device__ __forceinline__ double prox0(double v) { return v > 0.0 ? v : 0.0; }
+
 // ---- unfused element-wise steps of Alg. 2 (one call per operation)
 __global__ void k_prox(const double* __restrict__ Ht, const double* __restrict__ U, double* __restrict__ H, int64_t n) {
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n; x += (int64_t)gridDim.x * kT) {
-    const double v = Ht[x] - U[x];
-    H[x] = v > 0.0 ? v : 0.0;                  // Alg. 2 l.7 with the indicator of R_+
-  }
+  elemwise(n, [&](int64_t x) {                        // Alg. 2 l.7 with the indicator of R_+
+    const double2 h = ld2(Ht, x), u = ld2(U, x);
+    st2(H, x, prox0(h.x - u.x), prox0(h.y - u.y));
+  }, [&](int64_t x) { H[x] = prox0(Ht[x] - U[x]); });
 }
 __global__ void k_dual(const double* __restrict__ H, const double* __restrict__ Ht, double* __restrict__ U, int64_t n) {
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n; x += (int64_t)gridDim.x * kT)
-    U[x] = U[x] + H[x] - Ht[x];                // Alg. 2 l.8
+  elemwise(n, [&](int64_t x) {                        // Alg. 2 l.8
+    const double2 h = ld2(H, x), t = ld2(Ht, x), u = ld2(U, x);
+    st2(U, x, u.x + h.x - t.x, u.y + h.y - t.y);
+  }, [&](int64_t x) { U[x] = U[x] + H[x] - Ht[x]; });
 }
 
 __device__ __forceinline__ void block_store4(double a, double b, double c, double d, double* __restrict__ part) {
@@ -123,14 +140,20 @@ __device__ __forceinline__ void block_store4(double a, double b, double c, doubl
   }
   if (threadIdx.x < 4) part[blockIdx.x * 4 + threadIdx.x] = red[threadIdx.x][0];
 }
+__device__ __forceinline__ void acc4(double h, double ht, double h0, double u, double& r, double& s, double& nh,
+                                     double& nu) {
+  const double e1 = h - ht, e2 = h - h0;
+  r += e1 * e1; s += e2 * e2; nh += h * h; nu += u * u;
+}
 // residual sums of the baseline (the norms of Alg. 2 l.9, one pass over the four matrices)
 __global__ void k_resid(const double* __restrict__ H, const double* __restrict__ Ht, const double* __restrict__ H0,
                         const double* __restrict__ U, int64_t n, double* __restrict__ part) {
   double r = 0, s = 0, h = 0, u = 0;
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n; x += (int64_t)gridDim.x * kT) {
-    const double e1 = H[x] - Ht[x], e2 = H[x] - H0[x];
-    r += e1 * e1; s += e2 * e2; h += H[x] * H[x]; u += U[x] * U[x];
-  }
+  elemwise(n, [&](int64_t x) {
+    const double2 a = ld2(H, x), t = ld2(Ht, x), z = ld2(H0, x), v = ld2(U, x);
+    acc4(a.x, t.x, z.x, v.x, r, s, h, u);
+    acc4(a.y, t.y, z.y, v.y, r, s, h, u);
+  }, [&](int64_t x) { acc4(H[x], Ht[x], H0[x], U[x], r, s, h, u); });
   block_store4(r, s, h, u, part);
 }
 
@@ -139,23 +162,34 @@ __global__ void k_resid(const double* __restrict__ H, const double* __restrict__
 __global__ void k_fused_T(const double* __restrict__ M, const double* __restrict__ H, const double* __restrict__ U,
                           const double* __restrict__ consts, double* __restrict__ T, int64_t n) {
   const double rho = consts[1];
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n; x += (int64_t)gridDim.x * kT)
-    T[x] = M[x] + rho * (H[x] + U[x]);
+  elemwise(n, [&](int64_t x) {
+    const double2 m = ld2(M, x), h = ld2(H, x), u = ld2(U, x);
+    st2(T, x, m.x + rho * (h.x + u.x), m.y + rho * (h.y + u.y));
+  }, [&](int64_t x) { T[x] = M[x] + rho * (H[x] + U[x]); });
 }
 // prox + dual + residual partials in one pass; H0 is the incoming H (no copy)
+__device__ __forceinline__ void epi1(double ht, double h0, double u0, double& hn, double& un, double& r, double& s,
+                                     double& nh, double& nu) {
+  hn = prox0(ht - u0);
+  un = u0 + hn - ht;
+  acc4(hn, ht, h0, un, r, s, nh, nu);
+}
 __global__ void k_fused_epi(const double* __restrict__ Ht, double* __restrict__ H, double* __restrict__ U, int64_t n,
                             double* __restrict__ part) {
   double r = 0, s = 0, h = 0, u = 0;
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n; x += (int64_t)gridDim.x * kT) {
-    const double ht = Ht[x], h0 = H[x], u0 = U[x];
-    const double v = ht - u0;
-    const double hn = v > 0.0 ? v : 0.0;
-    const double un = u0 + hn - ht;
-    const double e1 = hn - ht, e2 = hn - h0;
-    r += e1 * e1; s += e2 * e2; h += hn * hn; u += un * un;
-    H[x] = hn;
-    U[x] = un;
-  }
+  elemwise(n, [&](int64_t x) {
+    const double2 t = ld2(Ht, x), h0 = ld2(H, x), u0 = ld2(U, x);
+    double a, b, c, d;
+    epi1(t.x, h0.x, u0.x, a, c, r, s, h, u);
+    epi1(t.y, h0.y, u0.y, b, d, r, s, h, u);
+    st2(H, x, a, b);
+    st2(U, x, c, d);
+  }, [&](int64_t x) {
+    double a, c;
+    epi1(Ht[x], H[x], U[x], a, c, r, s, h, u);
+    H[x] = a;
+    U[x] = c;
+  });
   block_store4(r, s, h, u, part);
 }
 
@@ -197,6 +231,7 @@ int cstf_ablation_admm(int arm, const double* d_M, const double* d_S, double* d_
   g_calls = 0;
   if (arm < CSTF_ABL_BASELINE || arm > CSTF_ABL_OF_PI) return err("unknown arm");
   if (R < 1 || R > 64 || I < 1 || max_iter < 1) return err("need R in [1, 64], I >= 1, max_iter >= 1");
+  if (((uintptr_t)d_M | (uintptr_t)d_H | (uintptr_t)d_U) & 15) return err("M, H, U must be 16-byte aligned");
   const bool fuse = arm == CSTF_ABL_OF || arm == CSTF_ABL_OF_PI;
   const bool pinv = arm == CSTF_ABL_PI || arm == CSTF_ABL_OF_PI;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -210,14 +245,15 @@ int cstf_ablation_admm(int arm, const double* d_M, const double* d_S, double* d_
   ABL(cublasSetStream(w.h, st));
   ABL(cublasSetPointerMode(w.h, CUBLAS_POINTER_MODE_DEVICE));
   const int64_t n = I * R;
-  const int nb = (int)std::min<int64_t>((n + kT - 1) / kT, (int64_t)sms * 4);
+  const int nb = (int)std::max<int64_t>(1, std::min<int64_t>((n / 2 + kT - 1) / kT, (int64_t)sms * 16));
   // workspace: Ht, T, H0 (I x R each), L, Inv (R x R), consts[4], partials, sums, flag
-  const size_t need = (size_t)(3 * n + 2 * R * R + 4 + nb * 4 + (size_t)max_iter * 4 + 2) * 8;
+  const int64_t np = (n + 1) & ~(int64_t)1;      // even offsets keep every matrix 16-byte aligned
+  const size_t need = (size_t)(3 * np + 2 * R * R + 4 + nb * 4 + (size_t)max_iter * 4 + 2) * 8;
   if (ensure(w, need)) return 1;
   double* Ht = static_cast<double*>(w.p);
-  double* Tb = Ht + n;
-  double* H0 = Tb + n;
-  double* Lc = H0 + n;
+  double* Tb = Ht + np;
+  double* H0 = Tb + np;
+  double* Lc = H0 + np;
   double* Inv = Lc + R * R;
   double* cst = Inv + R * R;
   double* part = cst + 4;

@@ -328,6 +328,20 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   // f4: fused all-gather through peer stores from the ADMM epilogue (falls back to
   // the NCCL / host all-gather when IPC mapping is unavailable or disabled)
   const bool peers = dist && open_peers(w, comm, st);
+  // hot-row tables (single GPU, factors >> L2): persisting set-aside for the whole call,
+  // released (and the caller's limit restored) on every return path
+  struct HotGuard {
+    L2Persist p;
+    cudaStream_t st;
+    ~HotGuard() {
+      if (p.active) {
+        cudaStreamSynchronize(st);
+        hot_persist_end(p);
+      }
+    }
+  } hotg;
+  hotg.st = st;
+  if (!dist) CSTF_TRY(hot_persist_begin(X, hotg.p));
   double* G = w.grams.as<double>();
   double* lam = w.lam.as<double>();
   double* lam_scratch = lam + (size_t)N * R;
@@ -361,6 +375,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       continue;
     }
     CSTF_TRY(init_factor(n, true));
+    CSTF_TRY(hot_refresh(X, n, fac[n], R, st));     // (no-op without hot rows)
   }
   if (peers) {   // no rank may peer-store into a replica another rank is still initialising / reading
     CSTF_TRY(comm_allreduce_f64(comm, w.xchg.as<double>(), 1, st));
@@ -406,7 +421,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       CSTF_CUDA(cudaEventRecord(w.join, w.side));
       // a2: MTTKRP of the raw factors (MTTKRP phase = both, overlapped)
       tm.begin(n, CSTF_PHASE_MTTKRP);
-      CSTF_TRY(mttkrp(X, n, R, fac.data(), M, st, nullptr));
+      CSTF_TRY(mttkrp(X, n, R, fac.data(), M, st, nullptr, /*hot_fresh=*/true));
       if (hin && t == 0 && n == 0) CSTF_TRY(init_factor(0, false));   // its copy overlapped MTTKRP(0)
       CSTF_CUDA(cudaStreamWaitEvent(st, w.join, 0));
       tm.end(n, CSTF_PHASE_MTTKRP);
@@ -448,6 +463,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       }
       if (rep && rep->admm_iters) rep->admm_iters[t * N + n] = iters;
       tm.end(n, CSTF_PHASE_UPDATE);
+      // the hot-row table of factor n follows its update (the next MTTKRPs read it)
+      if (!dist) CSTF_TRY(hot_refresh(X, n, Hn, R, st));
       // a7 (when not fused): raw Gram; a6: lambda and the normalised Gram
       if (!fused) {
         tm.begin(n, CSTF_PHASE_GRAM);

@@ -113,6 +113,9 @@ struct ModeStore {
   mutable DevBuf clb, ccont;
   mutable int64_t cchunk = -1, cnchunks = 0;
   mutable std::vector<int64_t> kp;   // L2-blocked copies: first nonzero of each block (host, cached)
+  // hot-row tables: bit q set = the records of slot q name hot rows of factor other[q]
+  // by (0x80000000 | hot slot)
+  int hotmask = 0;
 };
 inline int record_bytes(int N) { return ((4 * (N - 1) + 8) + 15) / 16 * 16; }
 
@@ -138,6 +141,15 @@ struct cstf_tensor {
   bool partitioned = false;           // loaded with a communicator (any size): row-partitioned layout
   int64_t rows_per_rank[8] = {0};     // B_n
   cstf::DevBuf relabel[8];            // int32[dims[n]]: internal label of original row
+  // Hot-row tables (single GPU, factors much larger than L2): the rows of factor k
+  // with the most nonzeros get hot slots hot_off[k] .. hot_off[k] + hot_cnt[k] - 1
+  // of one table (hot_total rows x R), refreshed from the factor and read by MTTKRP
+  // under a persisting L2 access window, so the L2 keeps exactly the rows most
+  // gathers hit.  hot_rows[hot slot] = factor row.
+  int64_t hot_cnt[8] = {0}, hot_off[8] = {0}, hot_total = 0;
+  cstf::DevBuf hot_rows;              // int32[hot_total]
+  mutable cstf::DevBuf hot_tab;       // hot_total x hot_R doubles (allocated on first use)
+  mutable int hot_R = 0;
 };
 
 namespace cstf {
@@ -149,8 +161,20 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
 cstf_status export_store(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals);
 
 // mttkrp.cu
+// hot_fresh: the hot-row tables already hold the current rows of every factor the
+// copy gathers (factorize refreshes them after each update); else they are refreshed
+// from d_factors first.
 cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d_factors,
-                   double* d_M, cudaStream_t st, int64_t* launches);
+                   double* d_M, cudaStream_t st, int64_t* launches, bool hot_fresh = false);
+// copy the hot rows of factor k (d_F, I_k x R) into X's hot table (allocated for R)
+cstf_status hot_refresh(const cstf_tensor* X, int k, const double* d_F, int R, cudaStream_t st);
+// persisting-L2 set-aside for the hot tables: set (saving the caller's) / restore + reset
+struct L2Persist {
+  size_t saved = 0;
+  bool active = false;
+};
+cstf_status hot_persist_begin(const cstf_tensor* X, L2Persist& p);
+void hot_persist_end(L2Persist& p);
 
 // dense.cu
 // G (R x R) = H^T H; if lam != nullptr also normalises: lam_r = sqrt(G_rr), H /= lam (in place),

@@ -45,6 +45,7 @@ struct MArgs {
   double* M;            // output rows (virtual rows when k-blocked)
   double* carry;        // [nchunks][R]
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
+  const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
 };
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
@@ -95,8 +96,9 @@ __device__ __forceinline__ const double2* row_addr(const char* base, unsigned j)
 // One warp processes chunk c.  Fb[q] = lane's byte offset into the row source of
 // slot q (a factor in global memory, or the shared-memory slab of a k-blocked
 // copy, already shifted by the slab's first row).
-template <int NOTHER, int R, int RECB, int GL = 0>
-__device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const char* const* Fb, int4* srec) {
+template <int NOTHER, int R, int RECB, int GL = 0, bool HOT = false>
+__device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const char* const* Fb, int4* srec,
+                                              const char* const* HFb = nullptr) {
   constexpr int RV = R / 2;                    // double2 per row
   constexpr int G = GL ? GL : (RV < 32 ? RV : 32);   // lanes per group
   constexpr int VPL = RV / G;                  // double2 per lane
@@ -177,7 +179,12 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
           double2 f[VPL];
 #pragma unroll
           for (int qq = 0; qq < NOTHER; qq++) {
-            const double2* rp = row_addr<ROWB>(Fb[qq], w[qq]);
+            const char* base = Fb[qq];
+            unsigned j = w[qq];
+            if constexpr (HOT) {            // hot row: its copy in the persisting hot-row table
+              if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
+            }
+            const double2* rp = row_addr<ROWB>(base, j);
 #pragma unroll
             for (int s = 0; s < VPL; s++) {
               const double2 x = rp[s * G];     // global (read-only) or shared slab
@@ -202,13 +209,18 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
 }
 
 // MINB: CTAs per SM the register budget targets (2 for long rows, 4 for short ones)
-template <int NOTHER, int R, int RECB, int MINB, int GL = 0>
+template <int NOTHER, int R, int RECB, int MINB, int GL = 0, bool HOT = false>
 __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
   constexpr int G = GL ? GL : ((R / 2) < 32 ? (R / 2) : 32);
   const int gl = (threadIdx.x & 31) % G;
   const char* Fb[NOTHER];
+  const char* HFb[HOT ? NOTHER : 1];
 #pragma unroll
   for (int q = 0; q < NOTHER; q++) Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
+  if constexpr (HOT) {
+#pragma unroll
+    for (int q = 0; q < NOTHER; q++) HFb[q] = reinterpret_cast<const char*>(a.HF[q] ? a.HF[q] : a.F[q]) + gl * 16;
+  }
   const int64_t warp0 = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5);
   const int64_t nwarps = (int64_t)gridDim.x * kWarps;
   __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
@@ -222,11 +234,11 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
       if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
       c = __shfl_sync(0xffffffffu, c, 0);
       if ((int64_t)c >= a.nchunks) break;
-      process_chunk<NOTHER, R, RECB, GL>(a, (int64_t)c, Fb, srec);
+      process_chunk<NOTHER, R, RECB, GL, HOT>(a, (int64_t)c, Fb, srec, HFb);
     }
     return;
   }
-  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL>(a, c, Fb, srec);
+  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT>(a, c, Fb, srec, HFb);
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -281,8 +293,10 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
         const double v = *reinterpret_cast<const double*>(r + a.recb - 8);
         double w[CPL];
         for (int q = 0; q < a.nother; q++) {
-          const unsigned j = reinterpret_cast<const unsigned*>(r)[q];
-          const double* src = a.F[q] + (size_t)j * (unsigned)R;
+          unsigned j = reinterpret_cast<const unsigned*>(r)[q];
+          const double* fq = a.F[q];
+          if ((int)j < 0) { fq = a.HF[q]; j &= 0x7fffffffu; }     // hot row (hot-row table)
+          const double* src = fq + (size_t)j * (unsigned)R;
 #pragma unroll
           for (int s = 0; s < CPL; s++) {
             const int col = lane + 32 * s;
@@ -393,7 +407,7 @@ bool launch_tiled_r(const MArgs& a, int grid, cudaStream_t st) {
 }
 
 template <int NOTHER, int RECB>
-bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl) {
+bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, bool hot) {
   // short rows (few nonzeros per row): row flushes dominate and latency hiding
   // needs more warps -> the 4-CTA/SM register budget; long rows -> 2 CTAs/SM
   const bool short_rows = a.nnz < 64 * (a.I - a.rbase);
@@ -414,6 +428,18 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl) 
   }
   GCASE(32, 8) GCASE(64, 16)
 #undef GCASE
+  if (hot) {           // copies with hot-row slots (large factors): R = 16 / 32 / 64, else generic
+    switch (a.R) {
+#define HCASE(RR)                                                                              \
+  case RR:                                                                                     \
+    if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4, 0, true><<<grid, kWarps * 32, 0, st>>>(a); \
+    else k_mttkrp_fast<NOTHER, RR, RECB, 2, 0, true><<<grid, kWarps * 32, 0, st>>>(a);           \
+    return true;
+      HCASE(16) HCASE(32) HCASE(64)
+#undef HCASE
+      default: return false;
+    }
+  }
   switch (a.R) {
 #define CASE(RR)                                                                     \
   case RR:                                                                           \
@@ -426,17 +452,18 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl) 
   }
 }
 
-cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, int gl) {
+cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, int gl, bool hot = false) {
   bool done = false;
   const bool tl = a.ckb != nullptr;
   const int g = tl ? tgrid : grid;
+  if (hot) gl = 0;                 // hot-row copies: the default group width (factors stream from HBM)
   switch (a.nother) {
-    case 1: done = launch_fast<1, 16>(a, grid, st, false, gl); break;
-    case 2: done = launch_fast<2, 16>(a, g, st, tl, gl); break;
-    case 3: done = launch_fast<3, 32>(a, g, st, tl, gl); break;
-    case 4: done = launch_fast<4, 32>(a, g, st, tl, gl); break;
-    case 5: done = launch_fast<5, 32>(a, g, st, tl, gl); break;
-    case 6: done = launch_fast<6, 32>(a, g, st, tl, gl); break;
+    case 1: done = launch_fast<1, 16>(a, grid, st, false, gl, hot); break;
+    case 2: done = launch_fast<2, 16>(a, g, st, tl, gl, hot); break;
+    case 3: done = launch_fast<3, 32>(a, g, st, tl, gl, hot); break;
+    case 4: done = launch_fast<4, 32>(a, g, st, tl, gl, hot); break;
+    case 5: done = launch_fast<5, 32>(a, g, st, tl, gl, hot); break;
+    case 6: done = launch_fast<6, 32>(a, g, st, tl, gl, hot); break;
     default: break;   // 7 other modes: 48-byte records, generic path
   }
   if (!done) {
@@ -513,7 +540,7 @@ cstf_status tiled_split(const ModeStore& ms, cudaStream_t st) {
 // blocked factor (its L2-resident slab); its partials continue the running sum of
 // M in block order.
 cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, double* d_M, cudaStream_t st,
-                              int64_t* nl) {
+                              int64_t* nl, bool hot) {
   const DeviceInfo& di = device_info();
   Workspace& w = ws();
   const int64_t I = ms.I, nblk = ms.nblk, nnz = ms.nnz;
@@ -637,7 +664,7 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
         if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v) != cudaSuccess) cudaGetLastError();
       }
       const int grid = (int)std::min<int64_t>((nchunks + kWarps - 1) / kWarps, (int64_t)ctas);
-      CSTF_TRY(launch_main(a, grid, grid, st, gl));
+      CSTF_TRY(launch_main(a, grid, grid, st, gl, hot));
       *nl += 2;
       if (nchunks > 1) {
         const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);
@@ -674,13 +701,64 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
 
 }  // namespace
 
+// tab[s, :] = F[rows[s], :] for the hot slots of one factor
+__global__ void k_hot_refresh(const double* __restrict__ F, const int32_t* __restrict__ rows, int64_t H, int R,
+                              double* __restrict__ tab) {
+  const int64_t n = H * R;
+  for (int64_t x = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; x < n; x += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t s = x / R, c = x % R;
+    tab[x] = F[(int64_t)rows[s] * R + c];
+  }
+}
+
+cstf_status hot_refresh(const cstf_tensor* X, int k, const double* d_F, int R, cudaStream_t st) {
+  if (X->hot_cnt[k] == 0) return CSTF_OK;
+  if (X->hot_R != R || !X->hot_tab.p) {
+    CSTF_TRY(X->hot_tab.alloc((size_t)X->hot_total * R * 8));
+    X->hot_R = R;
+  }
+  const int64_t n = X->hot_cnt[k] * R;
+  const int g = (int)std::min<int64_t>((n + 255) / 256, (int64_t)device_info().sms * 16);
+  k_hot_refresh<<<g, 256, 0, st>>>(d_F, X->hot_rows.as<int32_t>() + X->hot_off[k], X->hot_cnt[k], R,
+                                   X->hot_tab.as<double>() + X->hot_off[k] * R);
+  CSTF_LAUNCHED();
+  return CSTF_OK;
+}
+
+// The persisting-L2 set-aside the hot-row window needs: the device maximum (the
+// caller's limit is saved and restored by hot_persist_end, which also releases the
+// persisting lines; call it after a stream synchronisation).
+cstf_status hot_persist_begin(const cstf_tensor* X, L2Persist& p) {
+  p.active = false;
+  if (X->hot_total == 0 || (getenv("CSTF_HOT_WINDOW") && atoi(getenv("CSTF_HOT_WINDOW")) == 0)) return CSTF_OK;
+  int maxp = 0;
+  cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, device_info().device);
+  if (maxp <= 0 || cudaDeviceGetLimit(&p.saved, cudaLimitPersistingL2CacheSize) != cudaSuccess) {
+    cudaGetLastError();
+    return CSTF_OK;
+  }
+  if (p.saved != (size_t)maxp && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)maxp) != cudaSuccess) {
+    cudaGetLastError();               // not available (e.g. MIG): hot tables without persistence
+    return CSTF_OK;
+  }
+  p.active = true;
+  return CSTF_OK;
+}
+
+void hot_persist_end(L2Persist& p) {
+  if (!p.active) return;
+  if (cudaCtxResetPersistingL2Cache() != cudaSuccess) cudaGetLastError();
+  if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, p.saved) != cudaSuccess) cudaGetLastError();
+  p.active = false;
+}
+
 void release_mttkrp_ws() {
   Workspace& w = ws();
   for (DevBuf* b : {&w.lb, &w.cont, &w.carry, &w.gsum, &w.partial, &w.kbptr, &w.queue}) b->release();
 }
 
 cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d_factors,
-                   double* d_M, cudaStream_t st, int64_t* launches) {
+                   double* d_M, cudaStream_t st, int64_t* launches, bool hot_fresh) {
   const ModeStore& ms = X->mode[mode];
   const int N = X->N;
   const DeviceInfo& di = device_info();
@@ -702,6 +780,50 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor
   a.It_blk = X->partitioned ? (int64_t)X->nranks * X->rows_per_rank[ms.other[ms.tslot]] : X->dims[ms.other[ms.tslot]];
   a.R = R;
+  for (int q = 0; q < 7; q++) a.HF[q] = nullptr;
+  // Hot-row tables: refresh from the caller's factors unless the caller keeps them
+  // current (factorize), then read the hot rows under a persisting access window
+  // over the whole table (the caller's window is restored after the launches).
+  const bool hot = ms.hotmask != 0 && X->hot_total > 0;
+  L2Persist own;
+  cudaStreamAttrValue saved_win = {};
+  bool win_set = false;
+  if (hot) {
+    for (int q = 0; q < N - 1; q++)
+      if (ms.hotmask & (1 << q)) {
+        if (!hot_fresh || X->hot_R != R) CSTF_TRY(hot_refresh(X, ms.other[q], d_factors[ms.other[q]], R, st));
+      }
+    for (int q = 0; q < N - 1; q++)
+      if (ms.hotmask & (1 << q)) a.HF[q] = X->hot_tab.as<double>() + X->hot_off[ms.other[q]] * R;
+    if (!hot_fresh) CSTF_TRY(hot_persist_begin(X, own));
+    int maxw = 0;
+    cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, di.device);
+    const bool persist_on = hot_fresh ? !(getenv("CSTF_HOT_WINDOW") && atoi(getenv("CSTF_HOT_WINDOW")) == 0)
+                                      : own.active;
+    if (persist_on && maxw > 0 && cudaStreamGetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &saved_win) == cudaSuccess) {
+      cudaStreamAttrValue v = {};
+      v.accessPolicyWindow.base_ptr = X->hot_tab.p;
+      v.accessPolicyWindow.num_bytes = std::min<size_t>((size_t)X->hot_total * R * 8, (size_t)maxw);
+      v.accessPolicyWindow.hitRatio = 1.0f;
+      v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+      v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+      if (cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess) win_set = true;
+      else cudaGetLastError();
+    } else {
+      cudaGetLastError();
+    }
+  }
+  // after the launches: the caller's window back; a standalone call also releases the
+  // persisting lines and the set-aside (one host synchronisation)
+  auto hot_done = [&]() -> cstf_status {
+    if (win_set && cudaStreamSetAttribute(st, cudaStreamAttributeAccessPolicyWindow, &saved_win) != cudaSuccess)
+      cudaGetLastError();
+    if (own.active) {
+      CSTF_CUDA(cudaStreamSynchronize(st));
+      hot_persist_end(own);
+    }
+    return CSTF_OK;
+  };
   // Lanes per factor row: 8 lanes x 32 B (4 nonzeros per warp step) when the gathered
   // factors are L2-resident -- more nonzeros per load instruction, so adjacent
   // fiber nonzeros share L1 wavefronts (NELL-2 1.80 -> 1.63 ms per mode); the
@@ -717,7 +839,9 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   }
   int64_t nl = 0;
   if (ms.tiled && !ms.slab) {
-    CSTF_TRY(mttkrp_l2_blocked(ms, a, R, gl, d_M, st, &nl));
+    const cstf_status sb = mttkrp_l2_blocked(ms, a, R, gl, d_M, st, &nl, hot);
+    CSTF_TRY(hot_done());
+    CSTF_TRY(sb);
     if (launches) *launches += nl;
     return CSTF_OK;
   }
@@ -783,7 +907,11 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
       grid = std::min(grid, di.sms * (nnz < 64 * ms.Ivirt ? 4 : 2));
     }
   }
-  CSTF_TRY(launch_main(a, grid, tgrid, st, gl));
+  {
+    const cstf_status sl = launch_main(a, grid, tgrid, st, gl, hot);
+    CSTF_TRY(hot_done());
+    CSTF_TRY(sl);
+  }
   nl++;
   if (nchunks > 1) {
     const int g = (int)std::min<int64_t>((nchunks * 32 + 255) / 256, (int64_t)di.sms * 8);

@@ -273,11 +273,12 @@ __global__ void k_gather_shift(const int32_t* __restrict__ in, const uint32_t* _
 
 struct RecArgs {
   const int32_t* idx[7];   // slot q source index array (canonical order)
+  const int32_t* hmap[7] = {nullptr};  // slot q: factor row -> hot slot or -1 (null: no hot rows)
   int nslots;
   int recb;
 };
 
-// rec[p] = {idx[q][perm[p]] ..., vals[perm[p]]}
+// rec[p] = {idx[q][perm[p]] ..., vals[perm[p]]}; a hot row is stored as 0x80000000 | hot slot
 __global__ void k_make_records(RecArgs a, const double* __restrict__ vals, const uint32_t* __restrict__ perm,
                                int64_t n, char* __restrict__ rec) {
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
@@ -285,19 +286,35 @@ __global__ void k_make_records(RecArgs a, const double* __restrict__ vals, const
     const uint32_t src = perm[p];
     char* r = rec + p * a.recb;
     int32_t* ri = reinterpret_cast<int32_t*>(r);
-    for (int q = 0; q < a.nslots; q++) ri[q] = a.idx[q][src];
+    for (int q = 0; q < a.nslots; q++) {
+      int32_t v = a.idx[q][src];
+      if (a.hmap[q]) {
+        const int32_t h = a.hmap[q][v];
+        if (h >= 0) v = (int32_t)(0x80000000u | (uint32_t)h);
+      }
+      ri[q] = v;
+    }
     for (int q = a.nslots; q < (a.recb - 8) / 4; q++) ri[q] = 0;
     *reinterpret_cast<double*>(r + a.recb - 8) = vals[src];
   }
 }
 
+struct HotArgs {
+  const int32_t* rows = nullptr;   // hot slot -> factor row (all factors, concatenated)
+  int64_t off[7] = {0};            // slot q: first hot slot of its factor
+};
+
 // inverse of k_make_records for export: SoA arrays of the record slots + values
 __global__ void k_split_records(const char* __restrict__ rec, int recb, int nslots, int64_t n, OutArgs out,
-                                double* __restrict__ vals) {
+                                double* __restrict__ vals, HotArgs hot) {
   for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < n;
        p += (int64_t)gridDim.x * blockDim.x) {
     const char* r = rec + p * recb;
-    for (int q = 0; q < nslots; q++) out.idx[q][p] = reinterpret_cast<const int32_t*>(r)[q];
+    for (int q = 0; q < nslots; q++) {
+      int32_t v = reinterpret_cast<const int32_t*>(r)[q];
+      if (v < 0) v = hot.rows[hot.off[q] + (v & 0x7fffffff)];
+      out.idx[q][p] = v;
+    }
     vals[p] = *reinterpret_cast<const double*>(r + recb - 8);
   }
 }
@@ -496,6 +513,64 @@ cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int
   return CSTF_OK;
 }
 
+// Hot-row tables (single GPU).  A factor k whose
+// rows do not fit half the L2 even at R = 32 (I_k * 256 B > L2 / 2) gets hot slots for
+// its rows with the most nonzeros: at most half the device's persisting-L2 maximum
+// in rows of 256 B (so the hot rows two factors contribute to one MTTKRP fit the
+// set-aside), only rows with >= 2 nonzeros, ties by row index; slots are in
+// descending count order.  CSTF_HOT=0 disables; CSTF_HOT_ROWS=<n> forces n hot rows
+// per factor that has more than 2n rows (tests).  hmap[k] (device int32[I_k]) maps a
+// row to its hot slot or -1 and is used while the mode copies are built.
+cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap, cudaStream_t st) {
+  const int N = X->N;
+  X->hot_total = 0;
+  if (N < 3 || (getenv("CSTF_HOT") && atoi(getenv("CSTF_HOT")) == 0)) return CSTF_OK;
+  const char* fe = getenv("CSTF_HOT_ROWS");
+  const int64_t forced = fe ? atoll(fe) : 0;
+  int maxp = 0;
+  cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, device_info().device);
+  const int64_t per_factor = forced > 0 ? forced : (int64_t)maxp / 256 / 2;
+  if (per_factor < 1) return CSTF_OK;
+  std::vector<int32_t> all;
+  for (int k = 0; k < N; k++) {
+    X->hot_off[k] = (int64_t)all.size();
+    X->hot_cnt[k] = 0;
+    const int64_t I = X->dims[k];
+    const bool big = forced > 0 ? I > 2 * forced : I * 256 > (int64_t)device_info().l2 / 2;
+    if (!big || nout == 0) continue;
+    DevBuf cnt;
+    CSTF_TRY(cnt.alloc((size_t)I * 8));
+    CSTF_CUDA(cudaMemsetAsync(cnt.p, 0, (size_t)I * 8, st));
+    k_histogram<<<grid_for(nout), kThreads, 0, st>>>(c_idx[k].as<int32_t>(), nout, cnt.as<unsigned long long>());
+    CSTF_LAUNCHED();
+    std::vector<int64_t> counts((size_t)I);
+    CSTF_CUDA(cudaMemcpyAsync(counts.data(), cnt.p, (size_t)I * 8, cudaMemcpyDeviceToHost, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    std::vector<int32_t> order((size_t)I);
+    for (int64_t i = 0; i < I; i++) order[(size_t)i] = (int32_t)i;
+    const int64_t H = std::min<int64_t>(per_factor, I);
+    auto by_count = [&](int32_t a, int32_t b) { return counts[a] != counts[b] ? counts[a] > counts[b] : a < b; };
+    std::partial_sort(order.begin(), order.begin() + H, order.end(), by_count);
+    int64_t h = 0;
+    while (h < H && counts[(size_t)order[(size_t)h]] >= 2) h++;
+    if (h == 0) continue;
+    std::vector<int32_t> map((size_t)I, -1);
+    for (int64_t s = 0; s < h; s++) map[(size_t)order[(size_t)s]] = (int32_t)s;
+    CSTF_TRY(hmap[k].alloc((size_t)I * 4));
+    CSTF_CUDA(cudaMemcpyAsync(hmap[k].p, map.data(), (size_t)I * 4, cudaMemcpyHostToDevice, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+    all.insert(all.end(), order.begin(), order.begin() + h);
+    X->hot_cnt[k] = h;
+  }
+  X->hot_total = (int64_t)all.size();
+  if (X->hot_total) {
+    CSTF_TRY(X->hot_rows.alloc(all.size() * 4));
+    CSTF_CUDA(cudaMemcpyAsync(X->hot_rows.p, all.data(), all.size() * 4, cudaMemcpyHostToDevice, st));
+    CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  return CSTF_OK;
+}
+
 cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const double* host_vals,
                         int64_t n, cudaStream_t st) {
   const int N = X->N;
@@ -602,7 +677,11 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     memcpy(&X->hash, &hv[1], 8);
   }
   if (X->partitioned) return build_partitioned(X, c_idx, c_vals, nout, tmp, st);
-  // ---- 6. per-mode copies: sorted by (i_n, other modes by increasing length), AoS records
+  // ---- 6. hot rows of the factors much larger than L2 (single GPU)
+  DevBuf hmap[8];
+  static const bool kblock_env = getenv("CSTF_KBLOCK") && atoi(getenv("CSTF_KBLOCK")) > 0;
+  if (!kblock_env) CSTF_TRY(decide_hot(X, c_idx, nout, hmap, st));
+  // ---- 7. per-mode copies: sorted by (i_n, other modes by increasing length), AoS records
   const int recb = record_bytes(N);
   for (int n_ = 0; n_ < N; n_++) {
     ModeStore& ms = X->mode[n_];
@@ -662,6 +741,16 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
     ra.nslots = N - 1;
     ra.recb = recb;
     for (int q = 0; q < N - 1; q++) ra.idx[q] = c_idx[ms.other[q]].as<int32_t>();
+    // hot rows in every slot of the copy except the L2-blocked one (its slab is
+    // L2-resident by construction) and except copies whose blocks run under their own
+    // persisting window (>= 16M nonzeros per block, mttkrp.cu)
+    ms.hotmask = 0;
+    const bool slab_window = ms.tiled && !ms.slab && nout / std::max<int64_t>(ms.nblk, 1) >= ((int64_t)16 << 20);
+    for (int q = 0; q < N - 1 && !ms.slab && !slab_window; q++)
+      if (X->hot_cnt[ms.other[q]] > 0 && !(ms.tiled && q == ms.tslot)) {
+        ra.hmap[q] = hmap[ms.other[q]].as<int32_t>();
+        ms.hotmask |= 1 << q;
+      }
     if (nout) {
       k_make_records<<<grid_for(nout), kThreads, 0, st>>>(ra, c_vals.as<double>(), pm.as<uint32_t>(), nout,
                                                           ms.rec.as<char>());
@@ -689,7 +778,10 @@ cstf_status export_store(const cstf_tensor* X, int32_t* const* host_idx, double*
   OutArgs oa;
   oa.N = N - 1;
   for (int q = 0; q < N - 1; q++) oa.idx[q] = soa[ms.other[q]].as<int32_t>();
-  k_split_records<<<grid_for(n), kThreads, 0, st>>>(ms.rec.as<char>(), ms.recb, N - 1, n, oa, vals.as<double>());
+  HotArgs ha;
+  ha.rows = X->hot_rows.as<int32_t>();
+  for (int q = 0; q < N - 1; q++) ha.off[q] = X->hot_off[ms.other[q]];
+  k_split_records<<<grid_for(n), kThreads, 0, st>>>(ms.rec.as<char>(), ms.recb, N - 1, n, oa, vals.as<double>(), ha);
   CSTF_LAUNCHED();
   const int32_t* keys[8];
   for (int m = 0; m < N; m++) keys[m] = soa[m].as<int32_t>();

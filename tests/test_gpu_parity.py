@@ -676,3 +676,55 @@ def test_nonfinite_input_is_reported(B):
     with pytest.raises(B.CstfError) as e:
         B.cstf_factorize(X, F, cu(np.zeros(4)), B.make_opts(4, outer_iters=2, tol=1e-2))
     assert e.value.status in (B.CSTF_ERR_NUMERIC, B.CSTF_ERR_NOT_SPD)
+
+
+@pytest.mark.parametrize("R", [32, 16, 8, 64, 5])
+@pytest.mark.parametrize("window", ["1", "0"])
+def test_mttkrp_hot_row_tables(B, R, window, monkeypatch):
+    """Hot-row tables: records of the rows with the most nonzeros
+    point into a separate table refreshed from the factor and read under a persisting
+    L2 window.  Forced at small size (CSTF_HOT_ROWS): MTTKRP of every mode against the
+    oracle (fast kernels for R = 16/32/64, generic otherwise), with and without the
+    window, the export restores the canonical COO bit for bit, and the result is
+    bitwise the one of the store without hot rows."""
+    monkeypatch.setenv("CSTF_HOT_ROWS", "300")
+    monkeypatch.setenv("CSTF_HOT_WINDOW", window)
+    monkeypatch.setenv("CSTF_MTTKRP_G", "0")           # the same lane-group width with and without hot rows
+    dims = (90, 5000, 1200, 40)
+    idx, vals = datagen.coo(dims, (2, 2, 3, 1), 200_000, 51)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    gi, gv = X.export_coo()
+    assert np.array_equal(gv, ref.vals) and all(np.array_equal(a, b) for a, b in zip(gi, ref.idx))
+    monkeypatch.setenv("CSTF_HOT", "0")
+    Xp = B.cstf_tensor_load_coo(dims, idx, vals)
+    F = datagen.init_factors(dims, R, 9)
+    Fd = [cu(f) for f in F]
+    for n in range(4):
+        M = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        got = host(M).copy()
+        assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, n
+        Mp = cu(np.full((dims[n], R), np.nan))
+        B.cstf_mttkrp(Xp, n, Fd, Mp)
+        assert np.array_equal(got, host(Mp)), n
+    # a changed factor is picked up (standalone calls refresh the tables)
+    F2 = [f * 1.5 for f in F]
+    M = cu(np.full((dims[0], R), np.nan))
+    B.cstf_mttkrp(X, 0, [cu(f) for f in F2], M)
+    assert normwise(host(M), oracle.mttkrp(ref, 0, F2)) <= TOL
+
+
+@pytest.mark.parametrize("tol,R", [(1e-2, 16), (0.0, 32)])
+def test_factorize_hot_row_tables(B, tol, R, monkeypatch):
+    """factorize keeps the hot-row tables current after every update (forced hot rows)."""
+    monkeypatch.setenv("CSTF_HOT_ROWS", "200")
+    c = datagen.CONFIGS["delicious"].scaled(1000, nnz_factor=700)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, R, c.seed)
+    orc, gpu, F, lam = run_both(B, c.dims, idx, vals, R, start, outer=4, tol=tol)
+    n, tie = compare_iteration_counts(gpu["iters"], orc, tol if tol > 0 else 1e-2)
+    assert tie is None
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+    for a, b in zip(F, orc["factors"]):
+        assert normwise(a, b) <= 1e-6

@@ -46,6 +46,7 @@ struct MArgs {
   double* carry;        // [nchunks][R]
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
+  int async_mask;       // != 0: k_mttkrp_async with these slots copied by cp.async (R = 32)
 };
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
@@ -239,6 +240,227 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
     return;
   }
   for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT>(a, c, Fb, srec, HFb);
+}
+
+// ---------------------------------------------------------------------------------
+// Asynchronous-gather variant (R = 32, short rows).
+// With factors far larger than L2 the plain kernel is bound by memory latency, not
+// bandwidth: a warp keeps only the gathers of ~1-2 steps in flight (registers), so
+// Delicious mode 2 moves 41 GB in 11.8 ms (3.5 TB/s).  Here the rows of the "big"
+// slots (bigmask: factors that stream from HBM) are copied by cp.async (LDGSTS, no
+// registers held) into a per-warp shared-memory ring 16-32 nonzeros ahead of the
+// products: the record batch of 32 nonzeros is split in two halves; while one half
+// is multiplied, the copies of the next half are in flight (cp.async.wait_group 1).
+// A half-warp copies one 256-byte row per instruction (16 lanes x 16 B, coalesced).
+// The arithmetic, its order and the row / carry logic are those of process_chunk
+// (G = 16 lanes per row, P = 2 nonzeros per step): results are bit-identical.
+constexpr int kAsyncWarps = 4;
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;\n" ::); }
+
+template <int NOTHER, int RECB, bool HOT>
+__device__ __forceinline__ void process_chunk_async(const MArgs& a, int64_t c, const char* const* Fb,
+                                                    const char* const* HFb, int4* sr, double2* ring,
+                                                    int bigmask) {
+  constexpr int R = 32, RV = 16, G = 16, P = 2;
+  constexpr unsigned ROWB = R * 8;
+  constexpr int NW = RECB / 4;
+  constexpr int NV = RECB / 16;
+  const int lane = threadIdx.x & 31;
+  const int sg = lane / G, gl = lane % G;
+  int nbig = 0, bidx[NOTHER];
+#pragma unroll
+  for (int q = 0; q < NOTHER; q++) bidx[q] = ((bigmask >> q) & 1) ? nbig++ : -1;
+  // ring[slot t (0..31)][big slot b][RV double2]
+  const int64_t p0 = chunk_begin(a, c);
+  const int64_t p1 = chunk_end(a, c);
+  const int32_t ct = a.cont[c];
+  int64_t row = ct >= 0 ? (int64_t)ct : a.lb[c];
+  const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
+  double2 acc = make_double2(0.0, 0.0);
+  int64_t seg_end = (row < row_end) ? min(a.rowptr[row + 1], p1) : p1;
+  auto flush = [&](int64_t r) {
+    acc.x += __shfl_xor_sync(0xffffffffu, acc.x, 16);
+    acc.y += __shfl_xor_sync(0xffffffffu, acc.y, 16);
+    if (sg == 0) {
+      double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (r - a.rbase) * (int64_t)R;
+      reinterpret_cast<double2*>(dst)[gl] = acc;
+    }
+    acc = make_double2(0.0, 0.0);
+  };
+  // copies of the big-slot rows of 16 nonzeros: batch positions t0 .. t0+15 starting at
+  // nonzero pb0; the record of position t comes from `get(t, q)` (shared or registers)
+  auto issue = [&](int64_t pb0, int t0, auto get) {
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+      const int k = 2 * i + sg;                  // this half-warp's nonzero of the pair
+      const bool ok = pb0 + k < p1;
+#pragma unroll
+      for (int q = 0; q < NOTHER; q++) {
+        if (bidx[q] < 0) continue;
+        unsigned j = get(k, q);
+        const char* base = Fb[q];
+        if constexpr (HOT) {
+          if ((int)j < 0) { base = HFb[q]; j &= 0x7fffffffu; }
+        }
+        if (ok) cp_async16(ring + ((t0 + k) * nbig + bidx[q]) * RV + gl, row_addr<ROWB>(base, j));
+      }
+    }
+    cp_async_commit();
+  };
+  int4 nxt[NV];
+#pragma unroll
+  for (int k = 0; k < NV; k++)
+    nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
+                              : make_int4(0, 0, 0, 0);
+  auto word_of = [](const int4& v, int w) { return (unsigned)(w == 0 ? v.x : w == 1 ? v.y : w == 2 ? v.z : v.w); };
+  auto from_sr = [&](int t) { return [=](int k, int q) { return word_of(sr[(t + k) * NV + q / 4], q % 4); }; };
+  // prologue: batch 0 published, its two halves in flight
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < NV; k++) sr[lane * NV + k] = nxt[k];
+  __syncwarp();
+#pragma unroll
+  for (int k = 0; k < NV; k++)
+    nxt[k] = (p0 + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + 32 + lane) * RECB) + k)
+                                   : make_int4(0, 0, 0, 0);
+  issue(p0, 0, from_sr(0));
+  issue(p0 + 16, 16, from_sr(16));
+  for (int64_t pb = p0; pb < p1; pb += 32) {
+    const int nb = (int)min((int64_t)32, p1 - pb);
+    for (int half = 0; half < 2; half++) {
+      const int tlo = 16 * half, thi = min(16 * half + 16, nb);
+      cp_async_wait1();
+      __syncwarp();
+      int t = tlo;
+      while (t < thi) {
+        const int64_t p = pb + t;
+        if (p >= seg_end) {
+          flush(row);
+          row++;
+          seg_end = min(a.rowptr[row + 1], p1);
+          continue;
+        }
+        const int run = (int)min((int64_t)(thi - t), seg_end - p);
+#pragma unroll 4
+        for (int done = 0; done < run; done += P) {
+          const bool ok = (done + sg) < run;
+          const int src = ok ? t + done + sg : t + done;
+          unsigned w[NW];
+#pragma unroll
+          for (int k = 0; k < NV; k++) {
+            const int4 x = sr[src * NV + k];
+            w[4 * k] = x.x; w[4 * k + 1] = x.y; w[4 * k + 2] = x.z; w[4 * k + 3] = x.w;
+          }
+          const double v = ok ? __hiloint2double((int)w[NW - 1], (int)w[NW - 2]) : 0.0;
+          double2 f = make_double2(0.0, 0.0);
+#pragma unroll
+          for (int qq = 0; qq < NOTHER; qq++) {
+            double2 x;
+            if (bidx[qq] >= 0) {
+              x = ring[(src * nbig + bidx[qq]) * RV + gl];
+            } else {
+              const char* base = Fb[qq];
+              unsigned j = w[qq];
+              if constexpr (HOT) {
+                if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
+              }
+              x = *row_addr<ROWB>(base, j);
+            }
+            if (qq == 0) f = x;
+            else { f.x *= x.x; f.y *= x.y; }
+          }
+          acc.x = fma(v, f.x, acc.x);
+          acc.y = fma(v, f.y, acc.y);
+        }
+        t += run;
+      }
+      __syncwarp();            // every lane is done with this half's ring slots and records
+      if (half == 0) {         // next batch, first half: records still in registers
+        const int64_t pn = pb + 32;
+        issue(pn, 0, [&](int k, int q) { return (unsigned)__shfl_sync(0xffffffffu, (int)word_of(nxt[q / 4], q % 4), k); });
+      } else {                 // publish the next batch; its second half from shared memory
+#pragma unroll
+        for (int k = 0; k < NV; k++) sr[lane * NV + k] = nxt[k];
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < NV; k++)
+          nxt[k] = (pb + 64 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 64 + lane) * RECB) + k)
+                                         : make_int4(0, 0, 0, 0);
+        issue(pb + 48, 16, from_sr(16));
+      }
+    }
+  }
+  asm volatile("cp.async.wait_all;\n" ::);
+  __syncwarp();
+  while (row < row_end) {
+    flush(row);
+    row++;
+  }
+}
+
+template <int NOTHER, int RECB, bool HOT>
+__global__ void __launch_bounds__(kAsyncWarps * 32, 3) k_mttkrp_async(MArgs a, int bigmask) {
+  extern __shared__ int4 dsm[];
+  constexpr int NV = RECB / 16;
+  const int warp = threadIdx.x >> 5, gl = (threadIdx.x & 31) % 16;
+  int nbig = 0;
+  for (int q = 0; q < NOTHER; q++) nbig += (bigmask >> q) & 1;
+  int4* sr = dsm + warp * 32 * NV;
+  double2* ring = reinterpret_cast<double2*>(dsm + kAsyncWarps * 32 * NV) + (size_t)warp * 32 * nbig * 16;
+  const char* Fb[NOTHER];
+  const char* HFb[NOTHER];
+#pragma unroll
+  for (int q = 0; q < NOTHER; q++) {
+    Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
+    HFb[q] = reinterpret_cast<const char*>(a.HF[q] ? a.HF[q] : a.F[q]) + gl * 16;
+  }
+  if (a.queue) {
+    for (;;) {
+      unsigned long long c = 0;
+      if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if ((int64_t)c >= a.nchunks) break;
+      process_chunk_async<NOTHER, RECB, HOT>(a, (int64_t)c, Fb, HFb, sr, ring, bigmask);
+    }
+    return;
+  }
+  const int64_t nwarps = (int64_t)gridDim.x * kAsyncWarps;
+  for (int64_t c = blockIdx.x * (int64_t)kAsyncWarps + warp; c < a.nchunks; c += nwarps)
+    process_chunk_async<NOTHER, RECB, HOT>(a, c, Fb, HFb, sr, ring, bigmask);
+}
+
+size_t async_smem(int recb, int nbig) {
+  return (size_t)kAsyncWarps * 32 * recb + (size_t)kAsyncWarps * 32 * nbig * 256;
+}
+
+template <int NOTHER, int RECB>
+bool launch_async(const MArgs& a, int bigmask, bool hot, cudaStream_t st, int* grid_out) {
+  int nbig = 0;
+  for (int q = 0; q < NOTHER; q++) nbig += (bigmask >> q) & 1;
+  const size_t smem = async_smem(RECB, nbig);
+  static bool attr[2] = {false, false};
+  static int per_sm[2][8] = {{0}};
+  auto kern = hot ? k_mttkrp_async<NOTHER, RECB, true> : k_mttkrp_async<NOTHER, RECB, false>;
+  if (!attr[hot]) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)async_smem(RECB, NOTHER)) != cudaSuccess) { cudaGetLastError(); return false; }
+    attr[hot] = true;
+  }
+  if (!per_sm[hot][nbig]) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[hot][nbig], kern, kAsyncWarps * 32, smem) != cudaSuccess ||
+        per_sm[hot][nbig] < 1) { cudaGetLastError(); return false; }
+  }
+  const int64_t ctas = (a.nchunks + kAsyncWarps - 1) / kAsyncWarps;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(ctas, (int64_t)device_info().sms * per_sm[hot][nbig]));
+  kern<<<grid, kAsyncWarps * 32, smem, st>>>(a, bigmask);
+  if (grid_out) *grid_out = grid;
+  return true;
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -457,6 +679,20 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, in
   const bool tl = a.ckb != nullptr;
   const int g = tl ? tgrid : grid;
   if (hot) gl = 0;                 // hot-row copies: the default group width (factors stream from HBM)
+  if (a.async_mask && a.R == 32 && !tl) {
+    switch (a.nother) {
+      case 2: done = launch_async<2, 16>(a, a.async_mask, hot, st, nullptr); break;
+      case 3: done = launch_async<3, 32>(a, a.async_mask, hot, st, nullptr); break;
+      case 4: done = launch_async<4, 32>(a, a.async_mask, hot, st, nullptr); break;
+      case 5: done = launch_async<5, 32>(a, a.async_mask, hot, st, nullptr); break;
+      case 6: done = launch_async<6, 32>(a, a.async_mask, hot, st, nullptr); break;
+      default: break;
+    }
+    if (done) {
+      CSTF_LAUNCHED();
+      return CSTF_OK;
+    }
+  }
   switch (a.nother) {
     case 1: done = launch_fast<1, 16>(a, grid, st, false, gl, hot); break;
     case 2: done = launch_fast<2, 16>(a, g, st, tl, gl, hot); break;
@@ -769,6 +1005,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.wstart = nullptr;
   a.ckb = nullptr;
   a.queue = nullptr;
+  a.async_mask = 0;
   a.pbase = 0;
   a.cbase = 0;
   a.rbase = 0;
@@ -836,6 +1073,22 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
     const char* ge = getenv("CSTF_MTTKRP_G");        // read per call (tests force both paths)
     if (ge && (atoi(ge) == 0 || atoi(ge) == 8)) gl = atoi(ge);
+  }
+  // Asynchronous gathers (k_mttkrp_async): R = 32, short rows (the 4-CTA/SM launches,
+  // latency-bound when factors stream from HBM), for the slots whose factor does not
+  // fit a quarter of L2.  CSTF_MTTKRP_ASYNC=0 disables, =2 also allows long rows,
+  // =3 forces every slot and every row length (tests at small sizes).
+  a.async_mask = 0;
+  {
+    const char* ae = getenv("CSTF_MTTKRP_ASYNC");
+    const int amode = ae ? atoi(ae) : 1;
+    const bool short_rows = nnz < 64 * ms.Ivirt;
+    if (amode > 0 && R == 32 && N - 1 >= 2 && N - 1 <= 6 && !ms.slab && (short_rows || amode >= 2)) {
+      for (int q = 0; q < N - 1; q++) {
+        if (ms.tiled && q == ms.tslot && amode != 3) continue;   // the L2-blocked slot's slab is L2-resident
+        if (amode == 3 || X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) a.async_mask |= 1 << q;
+      }
+    }
   }
   int64_t nl = 0;
   if (ms.tiled && !ms.slab) {

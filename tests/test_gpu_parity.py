@@ -707,7 +707,10 @@ def test_mttkrp_hot_row_tables(B, R, window, monkeypatch):
         assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, n
         Mp = cu(np.full((dims[n], R), np.nan))
         B.cstf_mttkrp(Xp, n, Fd, Mp)
-        assert np.array_equal(got, host(Mp)), n
+        if R in (16, 32, 64):          # same fast kernel and order (other R: generic vs fast kernel)
+            assert np.array_equal(got, host(Mp)), n
+        else:
+            assert normwise(got, host(Mp)) <= TOL, n
     # a changed factor is picked up (standalone calls refresh the tables)
     F2 = [f * 1.5 for f in F]
     M = cu(np.full((dims[0], R), np.nan))
@@ -724,6 +727,54 @@ def test_factorize_hot_row_tables(B, tol, R, monkeypatch):
     start = datagen.init_factors(c.dims, R, c.seed)
     orc, gpu, F, lam = run_both(B, c.dims, idx, vals, R, start, outer=4, tol=tol)
     n, tie = compare_iteration_counts(gpu["iters"], orc, tol if tol > 0 else 1e-2)
+    assert tie is None
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+    for a, b in zip(F, orc["factors"]):
+        assert normwise(a, b) <= 1e-6
+
+
+@pytest.mark.parametrize("case", [("3mode", (300, 2111, 970), 200_000, (2, 2, 3)),
+                                  ("4mode", (90, 5000, 1200, 40), 200_000, (2, 2, 3, 1)),
+                                  ("2mode", (4000, 3000), 60_000, (2, 3)),
+                                  ("5mode", (30, 40, 50, 60, 20), 50_000, (2, 1, 2, 3, 1))])
+@pytest.mark.parametrize("hot", ["0", "150"])
+def test_mttkrp_async_gathers(B, case, hot, monkeypatch):
+    """k_mttkrp_async (cp.async row copies into a per-warp shared-memory ring, 16-32
+    nonzeros ahead of the products; R = 32) forced on every slot and mode
+    (CSTF_MTTKRP_ASYNC=3), with and without hot-row tables, against the oracle;
+    bitwise repeatable; rows without nonzeros stay zero."""
+    monkeypatch.setenv("CSTF_MTTKRP_ASYNC", "3")
+    if hot != "0":
+        monkeypatch.setenv("CSTF_HOT_ROWS", hot)
+    else:
+        monkeypatch.setenv("CSTF_HOT", "0")
+    name, dims, nnz, gam = case
+    idx, vals = datagen.coo(dims, gam, nnz, 61)
+    idx[0] = (idx[0] // 2 * 2).astype(np.int32)                 # odd rows of mode 0 empty
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    F = datagen.init_factors(dims, 32, 12)
+    Fd = [cu(f) for f in F]
+    for n in range(len(dims)):
+        M = cu(np.full((dims[n], 32), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        got = host(M).copy()
+        assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, (name, n)
+        B.cstf_mttkrp(X, n, Fd, M)
+        assert np.array_equal(host(M), got), (name, n)
+        if n == 0:
+            assert np.all(got[1::2] == 0.0)
+
+
+def test_factorize_async_gathers(B, monkeypatch):
+    """The factorisation with asynchronous gathers forced (and hot rows) vs the oracle."""
+    monkeypatch.setenv("CSTF_MTTKRP_ASYNC", "3")
+    monkeypatch.setenv("CSTF_HOT_ROWS", "200")
+    c = datagen.CONFIGS["delicious"].scaled(1000, nnz_factor=700)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, 32, c.seed)
+    orc, gpu, F, lam = run_both(B, c.dims, idx, vals, 32, start, outer=4, tol=1e-2)
+    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
     assert tie is None
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
     for a, b in zip(F, orc["factors"]):

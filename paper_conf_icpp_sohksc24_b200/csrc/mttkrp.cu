@@ -47,7 +47,28 @@ struct MArgs {
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
   int async_mask;       // != 0: k_mttkrp_async with these slots copied by cp.async (R = 32)
+  int pf_mask;          // slots whose rows are bulk-prefetched into L2 one record batch ahead
 };
+
+// L2 prefetch of the rows the next record batch gathers (DESIGN.md "MTTKRP, L2
+// prefetch"): lane L holds the record of nonzero pnext + L and issues one
+// cp.async.bulk.prefetch.L2 of the whole row per prefetched slot -- no registers or
+// shared memory held, 1 instruction per row, so the gathers of the batch after
+// the current one are in flight while this one multiplies.
+template <int NOTHER, int NV>
+__device__ __forceinline__ void prefetch_rows(const MArgs& a, const int4 (&rec)[NV], bool valid, int rowbytes) {
+  if (!a.pf_mask || !valid) return;
+#pragma unroll
+  for (int q = 0; q < NOTHER; q++) {
+    if (!((a.pf_mask >> q) & 1)) continue;
+    const int4 v = rec[q / 4];
+    unsigned j = (unsigned)((q % 4) == 0 ? v.x : (q % 4) == 1 ? v.y : (q % 4) == 2 ? v.z : v.w);
+    const double* base = a.F[q];
+    if ((int)j < 0) { base = a.HF[q]; j &= 0x7fffffffu; }
+    const char* addr = reinterpret_cast<const char*>(base) + (size_t)j * rowbytes;
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(addr), "r"(rowbytes) : "memory");
+  }
+}
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
 // nonzero range: a launch over a batch of L2 blocks splits every row exactly where
@@ -146,6 +167,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
     for (int k = 0; k < NV; k++)
       nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
                                 : make_int4(0, 0, 0, 0);
+    prefetch_rows<NOTHER, NV>(a, nxt, p0 + lane < p1, (int)ROWB);
     for (int64_t pb = p0; pb < p1; pb += 32) {
       const int nb = (int)min((int64_t)32, p1 - pb);
       __syncwarp();
@@ -156,6 +178,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
       for (int k = 0; k < NV; k++)
         nxt[k] = (pb + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 32 + lane) * RECB) + k)
                                        : make_int4(0, 0, 0, 0);
+      prefetch_rows<NOTHER, NV>(a, nxt, pb + 32 + lane < p1, (int)ROWB);
       int t = 0;
       while (t < nb) {
         const int64_t p = pb + t;
@@ -1006,6 +1029,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.ckb = nullptr;
   a.queue = nullptr;
   a.async_mask = 0;
+  a.pf_mask = 0;
   a.pbase = 0;
   a.cbase = 0;
   a.rbase = 0;
@@ -1076,12 +1100,13 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   }
   // Asynchronous gathers (k_mttkrp_async): R = 32, short rows (the 4-CTA/SM launches,
   // latency-bound when factors stream from HBM), for the slots whose factor does not
-  // fit a quarter of L2.  CSTF_MTTKRP_ASYNC=0 disables, =2 also allows long rows,
+  // fit a quarter of L2.  Off by default (measured slower than the L2 prefetch below:
+  // DESIGN.md); CSTF_MTTKRP_ASYNC=1 enables it for short rows, =2 also for long rows,
   // =3 forces every slot and every row length (tests at small sizes).
   a.async_mask = 0;
   {
     const char* ae = getenv("CSTF_MTTKRP_ASYNC");
-    const int amode = ae ? atoi(ae) : 1;
+    const int amode = ae ? atoi(ae) : 0;      // off by default: slower than the L2 prefetch
     const bool short_rows = nnz < 64 * ms.Ivirt;
     if (amode > 0 && R == 32 && N - 1 >= 2 && N - 1 <= 6 && !ms.slab && (short_rows || amode >= 2)) {
       for (int q = 0; q < N - 1; q++) {
@@ -1089,6 +1114,18 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
         if (amode == 3 || X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) a.async_mask |= 1 << q;
       }
     }
+  }
+  // L2 prefetch one record batch ahead for the slots whose factor does not fit a
+  // quarter of L2 (they stream from HBM; the kernel is bound by their latency).
+  // CSTF_MTTKRP_PF=0 disables, =2 forces every slot (tests).
+  {
+    const char* pe = getenv("CSTF_MTTKRP_PF");
+    const int pmode = pe ? atoi(pe) : 1;
+    if (pmode > 0 && !ms.slab && a.async_mask == 0)
+      for (int q = 0; q < N - 1; q++) {
+        if (ms.tiled && q == ms.tslot && pmode != 2) continue;
+        if (pmode == 2 || X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) a.pf_mask |= 1 << q;
+      }
   }
   int64_t nl = 0;
   if (ms.tiled && !ms.slab) {

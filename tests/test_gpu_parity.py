@@ -738,12 +738,15 @@ def test_factorize_hot_row_tables(B, tol, R, monkeypatch):
                                   ("2mode", (4000, 3000), 60_000, (2, 3)),
                                   ("5mode", (30, 40, 50, 60, 20), 50_000, (2, 1, 2, 3, 1))])
 @pytest.mark.parametrize("hot", ["0", "150"])
-def test_mttkrp_async_gathers(B, case, hot, monkeypatch):
+@pytest.mark.parametrize("knob", ["CSTF_MTTKRP_ASYNC=3", "CSTF_MTTKRP_PF=2"])
+def test_mttkrp_async_gathers(B, case, hot, knob, monkeypatch):
     """k_mttkrp_async (cp.async row copies into a per-warp shared-memory ring, 16-32
     nonzeros ahead of the products; R = 32) forced on every slot and mode
     (CSTF_MTTKRP_ASYNC=3), with and without hot-row tables, against the oracle;
-    bitwise repeatable; rows without nonzeros stay zero."""
-    monkeypatch.setenv("CSTF_MTTKRP_ASYNC", "3")
+    bitwise repeatable; rows without nonzeros stay zero.  The same checks for the
+    L2 bulk prefetch of the next record batch's rows forced on every slot."""
+    k, v = knob.split("=")
+    monkeypatch.setenv(k, v)
     if hot != "0":
         monkeypatch.setenv("CSTF_HOT_ROWS", hot)
     else:

@@ -48,6 +48,7 @@ struct MArgs {
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
   int async_mask;       // != 0: k_mttkrp_async with these slots copied by cp.async (R = 32)
   int pf_mask;          // slots whose rows are bulk-prefetched into L2 one record batch ahead
+  int flat;             // != 0: k_mttkrp_flat (one nonzero per warp step, loads independent of rows)
 };
 
 // L2 prefetch of the rows the next record batch gathers (DESIGN.md "MTTKRP, L2
@@ -263,6 +264,161 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
     return;
   }
   for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT>(a, c, Fb, srec, HFb);
+}
+
+// ---------------------------------------------------------------------------------
+// Flat-stream variant (R = 32 / 64).  The plain
+// kernel walks a chunk row by row: the gathers of a row's nonzeros are issued, the
+// row is reduced and stored, and only then do the next row's gathers start -- with
+// 8 nonzeros per row (Delicious mode 2) every row costs a full HBM round trip per
+// warp, and the kernel is latency-bound at half the HBM rate.  Here all 32 lanes
+// work on ONE nonzero per step (R/32 doubles each, no cross-lane reduction) and the
+// gathers of U consecutive nonzeros are issued together whatever rows they belong
+// to; rows are then closed in order.  Row membership comes from a window of 32 row
+// ends (lane L holds the end of row wrow + L): the row of nonzero p is
+// wrow + popc(ballot(end <= p)).  Chunk / carry logic as in process_chunk.
+template <int NOTHER, int R, int RECB, bool HOT, int U>
+__device__ __forceinline__ void process_chunk_flat(const MArgs& a, int64_t c, int4* sr) {
+  constexpr int VD = R / 32;                   // doubles per lane
+  constexpr int NV = RECB / 16;
+  constexpr int NW = RECB / 4;
+  const int lane = threadIdx.x & 31;
+  const int64_t p0 = chunk_begin(a, c);
+  const int64_t p1 = chunk_end(a, c);
+  const int32_t ct = a.cont[c];
+  const int64_t row0 = ct >= 0 ? (int64_t)ct : a.lb[c];
+  const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
+  double acc[VD];
+#pragma unroll
+  for (int i = 0; i < VD; i++) acc[i] = 0.0;
+  int64_t cur = row0;
+  int64_t wrow = row0;
+  int64_t e = 0;
+  auto load_window = [&]() {
+    const int64_t r = wrow + lane;
+    e = (r < row_end - 1) ? a.rowptr[r + 1] : INT64_MAX;   // the chunk's last row ends at or after p1
+  };
+  auto flush = [&](int64_t r) {
+    double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (r - a.rbase) * (int64_t)R;
+    if constexpr (VD == 2) reinterpret_cast<double2*>(dst)[lane] = make_double2(acc[0], acc[1]);
+    else dst[lane] = acc[0];
+#pragma unroll
+    for (int i = 0; i < VD; i++) acc[i] = 0.0;
+  };
+  load_window();
+  int4* srw = sr + (threadIdx.x >> 5) * 32 * NV;
+  int4 nxt[NV];
+#pragma unroll
+  for (int k = 0; k < NV; k++)
+    nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
+                              : make_int4(0, 0, 0, 0);
+  for (int64_t pb = p0; pb < p1; pb += 32) {
+    const int nb = (int)min((int64_t)32, p1 - pb);
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < NV; k++) srw[lane * NV + k] = nxt[k];
+    __syncwarp();
+#pragma unroll
+    for (int k = 0; k < NV; k++)
+      nxt[k] = (pb + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 32 + lane) * RECB) + k)
+                                     : make_int4(0, 0, 0, 0);
+    for (int t = 0; t < nb; t += U) {
+      double x[U][NOTHER][VD];
+      double v[U];
+      // gathers of U nonzeros, issued together (independent of their rows)
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        v[u] = 0.0;
+        if (t + u < nb) {
+          const int4* rc = srw + (t + u) * NV;
+          const int4 r0 = rc[0];
+          const int4 rv = rc[NV - 1];
+          v[u] = __hiloint2double(NV == 1 ? r0.w : rv.w, NV == 1 ? r0.z : rv.z);
+          unsigned w[NOTHER];
+#pragma unroll
+          for (int q = 0; q < NOTHER; q++) {
+            const int4 rq = rc[q / 4];
+            w[q] = (unsigned)((q % 4) == 0 ? rq.x : (q % 4) == 1 ? rq.y : (q % 4) == 2 ? rq.z : rq.w);
+          }
+#pragma unroll
+          for (int q = 0; q < NOTHER; q++) {
+            const double* base = a.F[q];
+            unsigned j = w[q];
+            if constexpr (HOT) {
+              if ((int)j < 0) { base = a.HF[q]; j &= 0x7fffffffu; }
+            }
+            const double* rp = base + (size_t)j * R + lane * VD;
+            if constexpr (VD == 2) {
+              const double2 y = *reinterpret_cast<const double2*>(rp);
+              x[u][q][0] = y.x; x[u][q][1] = y.y;
+            } else {
+              x[u][q][0] = *rp;
+            }
+          }
+        }
+      }
+      // rows closed in order, then the products accumulated
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        if (t + u >= nb) break;
+        const int64_t p = pb + t + u;
+        unsigned m = __ballot_sync(0xffffffffu, e <= p);
+        while (m == 0xffffffffu) {             // 32 rows of the window ended: slide it
+          while (cur < wrow + 32) { flush(cur); cur++; }
+          wrow += 32;
+          load_window();
+          m = __ballot_sync(0xffffffffu, e <= p);
+        }
+        const int64_t rp = wrow + __popc(m);
+        while (cur < rp) { flush(cur); cur++; }
+#pragma unroll
+        for (int i = 0; i < VD; i++) {
+          double f = x[u][0][i];
+#pragma unroll
+          for (int q = 1; q < NOTHER; q++) f *= x[u][q][i];
+          acc[i] = fma(v[u], f, acc[i]);
+        }
+      }
+    }
+  }
+  while (cur < row_end) { flush(cur); cur++; }
+}
+
+template <int NOTHER, int R, int RECB, bool HOT, int MINB = 4>
+__global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_flat(MArgs a) {
+  __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
+  if (a.queue) {
+    for (;;) {
+      unsigned long long c = 0;
+      if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
+      c = __shfl_sync(0xffffffffu, c, 0);
+      if ((int64_t)c >= a.nchunks) break;
+      process_chunk_flat<NOTHER, R, RECB, HOT, 4>(a, (int64_t)c, srec);
+    }
+    return;
+  }
+  const int64_t nwarps = (int64_t)gridDim.x * kWarps;
+  for (int64_t c = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5); c < a.nchunks; c += nwarps)
+    process_chunk_flat<NOTHER, R, RECB, HOT, 4>(a, c, srec);
+}
+
+template <int NOTHER, int RECB>
+bool launch_flat(const MArgs& a, bool hot, int grid, cudaStream_t st) {
+  const char* me = getenv("CSTF_MTTKRP_FLAT_MINB");      // 3: 85 registers, 3 CTAs/SM (experiments)
+  const bool m3 = me && atoi(me) == 3;
+  if (m3) grid = std::min(grid, device_info().sms * 3);
+#define FCASE(RR)                                                                          \
+  if (a.R == RR) {                                                                          \
+    if (m3) {                                                                               \
+      if (hot) k_mttkrp_flat<NOTHER, RR, RECB, true, 3><<<grid, kWarps * 32, 0, st>>>(a);  \
+      else k_mttkrp_flat<NOTHER, RR, RECB, false, 3><<<grid, kWarps * 32, 0, st>>>(a);     \
+    } else if (hot) k_mttkrp_flat<NOTHER, RR, RECB, true><<<grid, kWarps * 32, 0, st>>>(a); \
+    else k_mttkrp_flat<NOTHER, RR, RECB, false><<<grid, kWarps * 32, 0, st>>>(a);          \
+    return true;                                                                            \
+  }
+  FCASE(32) FCASE(64)
+#undef FCASE
+  return false;
 }
 
 // ---------------------------------------------------------------------------------
@@ -702,6 +858,21 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, in
   const bool tl = a.ckb != nullptr;
   const int g = tl ? tgrid : grid;
   if (hot) gl = 0;                 // hot-row copies: the default group width (factors stream from HBM)
+  if (a.flat && !tl && (a.R == 32 || a.R == 64)) {
+    const int fg = std::min(grid, device_info().sms * 4);
+    switch (a.nother) {
+      case 2: done = launch_flat<2, 16>(a, hot, fg, st); break;
+      case 3: done = launch_flat<3, 32>(a, hot, fg, st); break;
+      case 4: done = launch_flat<4, 32>(a, hot, fg, st); break;
+      case 5: done = launch_flat<5, 32>(a, hot, fg, st); break;
+      case 6: done = launch_flat<6, 32>(a, hot, fg, st); break;
+      default: break;
+    }
+    if (done) {
+      CSTF_LAUNCHED();
+      return CSTF_OK;
+    }
+  }
   if (a.async_mask && a.R == 32 && !tl) {
     switch (a.nother) {
       case 2: done = launch_async<2, 16>(a, a.async_mask, hot, st, nullptr); break;
@@ -1030,6 +1201,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.queue = nullptr;
   a.async_mask = 0;
   a.pf_mask = 0;
+  a.flat = 0;
   a.pbase = 0;
   a.cbase = 0;
   a.rbase = 0;
@@ -1115,12 +1287,28 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
       }
     }
   }
+  // Flat stream (k_mttkrp_flat): R = 32 / 64 short-row copies that gather a factor
+  // larger than L2/4 (latency-bound).  CSTF_MTTKRP_FLAT=0 disables, =2 forces it
+  // for every R = 32 / 64 launch (tests).
+  {
+    const char* fe = getenv("CSTF_MTTKRP_FLAT");
+    const int fmode = fe ? atoi(fe) : 1;
+    const bool short_rows = nnz < 64 * ms.Ivirt;
+    bool big = false;
+    for (int q = 0; q < N - 1; q++)
+      if (!(ms.tiled && q == ms.tslot) && X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) big = true;
+    if ((R == 32 || R == 64) && N - 1 >= 2 && N - 1 <= 6 && !ms.slab && a.async_mask == 0 &&
+        ((fmode == 1 && short_rows && big) || fmode == 2))
+      a.flat = 1;
+  }
   // L2 prefetch one record batch ahead for the slots whose factor does not fit a
-  // quarter of L2 (they stream from HBM; the kernel is bound by their latency).
-  // CSTF_MTTKRP_PF=0 disables, =2 forces every slot (tests).
+  // quarter of L2.  Off by default: measured slower (Delicious mode 0 9.4 -> 16 ms,
+  // DRAM reads 58 -> 108 GB: with ~4,700 warps each 32 nonzeros ahead, 77 MB of
+  // prefetched rows are in flight and evict each other before use).
+  // CSTF_MTTKRP_PF=1 enables it for those slots, =2 for every slot (tests).
   {
     const char* pe = getenv("CSTF_MTTKRP_PF");
-    const int pmode = pe ? atoi(pe) : 1;
+    const int pmode = pe ? atoi(pe) : 0;
     if (pmode > 0 && !ms.slab && a.async_mask == 0)
       for (int q = 0; q < N - 1; q++) {
         if (ms.tiled && q == ms.tslot && pmode != 2) continue;

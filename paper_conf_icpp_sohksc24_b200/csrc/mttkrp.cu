@@ -46,30 +46,7 @@ struct MArgs {
   double* carry;        // [nchunks][R]
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
-  int async_mask;       // != 0: k_mttkrp_async with these slots copied by cp.async (R = 32)
-  int pf_mask;          // slots whose rows are bulk-prefetched into L2 one record batch ahead
-  int flat;             // != 0: k_mttkrp_flat (one nonzero per warp step, loads independent of rows)
 };
-
-// L2 prefetch of the rows the next record batch gathers (DESIGN.md "MTTKRP, L2
-// prefetch"): lane L holds the record of nonzero pnext + L and issues one
-// cp.async.bulk.prefetch.L2 of the whole row per prefetched slot -- no registers or
-// shared memory held, 1 instruction per row, so the gathers of the batch after
-// the current one are in flight while this one multiplies.
-template <int NOTHER, int NV>
-__device__ __forceinline__ void prefetch_rows(const MArgs& a, const int4 (&rec)[NV], bool valid, int rowbytes) {
-  if (!a.pf_mask || !valid) return;
-#pragma unroll
-  for (int q = 0; q < NOTHER; q++) {
-    if (!((a.pf_mask >> q) & 1)) continue;
-    const int4 v = rec[q / 4];
-    unsigned j = (unsigned)((q % 4) == 0 ? v.x : (q % 4) == 1 ? v.y : (q % 4) == 2 ? v.z : v.w);
-    const double* base = a.F[q];
-    if ((int)j < 0) { base = a.HF[q]; j &= 0x7fffffffu; }
-    const char* addr = reinterpret_cast<const char*>(base) + (size_t)j * rowbytes;
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(addr), "r"(rowbytes) : "memory");
-  }
-}
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
 // nonzero range: a launch over a batch of L2 blocks splits every row exactly where
@@ -168,7 +145,6 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
     for (int k = 0; k < NV; k++)
       nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
                                 : make_int4(0, 0, 0, 0);
-    prefetch_rows<NOTHER, NV>(a, nxt, p0 + lane < p1, (int)ROWB);
     for (int64_t pb = p0; pb < p1; pb += 32) {
       const int nb = (int)min((int64_t)32, p1 - pb);
       __syncwarp();
@@ -179,7 +155,6 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
       for (int k = 0; k < NV; k++)
         nxt[k] = (pb + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 32 + lane) * RECB) + k)
                                        : make_int4(0, 0, 0, 0);
-      prefetch_rows<NOTHER, NV>(a, nxt, pb + 32 + lane < p1, (int)ROWB);
       int t = 0;
       while (t < nb) {
         const int64_t p = pb + t;
@@ -264,382 +239,6 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
     return;
   }
   for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT>(a, c, Fb, srec, HFb);
-}
-
-// ---------------------------------------------------------------------------------
-// Flat-stream variant (R = 32 / 64).  The plain
-// kernel walks a chunk row by row: the gathers of a row's nonzeros are issued, the
-// row is reduced and stored, and only then do the next row's gathers start -- with
-// 8 nonzeros per row (Delicious mode 2) every row costs a full HBM round trip per
-// warp, and the kernel is latency-bound at half the HBM rate.  Here all 32 lanes
-// work on ONE nonzero per step (R/32 doubles each, no cross-lane reduction) and the
-// gathers of U consecutive nonzeros are issued together whatever rows they belong
-// to; rows are then closed in order.  Row membership comes from a window of 32 row
-// ends (lane L holds the end of row wrow + L): the row of nonzero p is
-// wrow + popc(ballot(end <= p)).  Chunk / carry logic as in process_chunk.
-template <int NOTHER, int R, int RECB, bool HOT, int U>
-__device__ __forceinline__ void process_chunk_flat(const MArgs& a, int64_t c, int4* sr) {
-  constexpr int VD = R / 32;                   // doubles per lane
-  constexpr int NV = RECB / 16;
-  constexpr int NW = RECB / 4;
-  const int lane = threadIdx.x & 31;
-  const int64_t p0 = chunk_begin(a, c);
-  const int64_t p1 = chunk_end(a, c);
-  const int32_t ct = a.cont[c];
-  const int64_t row0 = ct >= 0 ? (int64_t)ct : a.lb[c];
-  const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
-  double acc[VD];
-#pragma unroll
-  for (int i = 0; i < VD; i++) acc[i] = 0.0;
-  int64_t cur = row0;
-  int64_t wrow = row0;
-  int64_t e = 0;
-  auto load_window = [&]() {
-    const int64_t r = wrow + lane;
-    e = (r < row_end - 1) ? a.rowptr[r + 1] : INT64_MAX;   // the chunk's last row ends at or after p1
-  };
-  auto flush = [&](int64_t r) {
-    double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (r - a.rbase) * (int64_t)R;
-    if constexpr (VD == 2) reinterpret_cast<double2*>(dst)[lane] = make_double2(acc[0], acc[1]);
-    else dst[lane] = acc[0];
-#pragma unroll
-    for (int i = 0; i < VD; i++) acc[i] = 0.0;
-  };
-  load_window();
-  int4* srw = sr + (threadIdx.x >> 5) * 32 * NV;
-  int4 nxt[NV];
-#pragma unroll
-  for (int k = 0; k < NV; k++)
-    nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
-                              : make_int4(0, 0, 0, 0);
-  for (int64_t pb = p0; pb < p1; pb += 32) {
-    const int nb = (int)min((int64_t)32, p1 - pb);
-    __syncwarp();
-#pragma unroll
-    for (int k = 0; k < NV; k++) srw[lane * NV + k] = nxt[k];
-    __syncwarp();
-#pragma unroll
-    for (int k = 0; k < NV; k++)
-      nxt[k] = (pb + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 32 + lane) * RECB) + k)
-                                     : make_int4(0, 0, 0, 0);
-    for (int t = 0; t < nb; t += U) {
-      double x[U][NOTHER][VD];
-      double v[U];
-      // gathers of U nonzeros, issued together (independent of their rows)
-#pragma unroll
-      for (int u = 0; u < U; u++) {
-        v[u] = 0.0;
-        if (t + u < nb) {
-          const int4* rc = srw + (t + u) * NV;
-          const int4 r0 = rc[0];
-          const int4 rv = rc[NV - 1];
-          v[u] = __hiloint2double(NV == 1 ? r0.w : rv.w, NV == 1 ? r0.z : rv.z);
-          unsigned w[NOTHER];
-#pragma unroll
-          for (int q = 0; q < NOTHER; q++) {
-            const int4 rq = rc[q / 4];
-            w[q] = (unsigned)((q % 4) == 0 ? rq.x : (q % 4) == 1 ? rq.y : (q % 4) == 2 ? rq.z : rq.w);
-          }
-#pragma unroll
-          for (int q = 0; q < NOTHER; q++) {
-            const double* base = a.F[q];
-            unsigned j = w[q];
-            if constexpr (HOT) {
-              if ((int)j < 0) { base = a.HF[q]; j &= 0x7fffffffu; }
-            }
-            const double* rp = base + (size_t)j * R + lane * VD;
-            if constexpr (VD == 2) {
-              const double2 y = *reinterpret_cast<const double2*>(rp);
-              x[u][q][0] = y.x; x[u][q][1] = y.y;
-            } else {
-              x[u][q][0] = *rp;
-            }
-          }
-        }
-      }
-      // rows closed in order, then the products accumulated
-#pragma unroll
-      for (int u = 0; u < U; u++) {
-        if (t + u >= nb) break;
-        const int64_t p = pb + t + u;
-        unsigned m = __ballot_sync(0xffffffffu, e <= p);
-        while (m == 0xffffffffu) {             // 32 rows of the window ended: slide it
-          while (cur < wrow + 32) { flush(cur); cur++; }
-          wrow += 32;
-          load_window();
-          m = __ballot_sync(0xffffffffu, e <= p);
-        }
-        const int64_t rp = wrow + __popc(m);
-        while (cur < rp) { flush(cur); cur++; }
-#pragma unroll
-        for (int i = 0; i < VD; i++) {
-          double f = x[u][0][i];
-#pragma unroll
-          for (int q = 1; q < NOTHER; q++) f *= x[u][q][i];
-          acc[i] = fma(v[u], f, acc[i]);
-        }
-      }
-    }
-  }
-  while (cur < row_end) { flush(cur); cur++; }
-}
-
-template <int NOTHER, int R, int RECB, bool HOT, int MINB = 4>
-__global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_flat(MArgs a) {
-  __shared__ int4 srec[kWarps * 32 * (RECB / 16)];
-  if (a.queue) {
-    for (;;) {
-      unsigned long long c = 0;
-      if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
-      c = __shfl_sync(0xffffffffu, c, 0);
-      if ((int64_t)c >= a.nchunks) break;
-      process_chunk_flat<NOTHER, R, RECB, HOT, 4>(a, (int64_t)c, srec);
-    }
-    return;
-  }
-  const int64_t nwarps = (int64_t)gridDim.x * kWarps;
-  for (int64_t c = blockIdx.x * (int64_t)kWarps + (threadIdx.x >> 5); c < a.nchunks; c += nwarps)
-    process_chunk_flat<NOTHER, R, RECB, HOT, 4>(a, c, srec);
-}
-
-template <int NOTHER, int RECB>
-bool launch_flat(const MArgs& a, bool hot, int grid, cudaStream_t st) {
-  const char* me = getenv("CSTF_MTTKRP_FLAT_MINB");      // 3: 85 registers, 3 CTAs/SM (experiments)
-  const bool m3 = me && atoi(me) == 3;
-  if (m3) grid = std::min(grid, device_info().sms * 3);
-#define FCASE(RR)                                                                          \
-  if (a.R == RR) {                                                                          \
-    if (m3) {                                                                               \
-      if (hot) k_mttkrp_flat<NOTHER, RR, RECB, true, 3><<<grid, kWarps * 32, 0, st>>>(a);  \
-      else k_mttkrp_flat<NOTHER, RR, RECB, false, 3><<<grid, kWarps * 32, 0, st>>>(a);     \
-    } else if (hot) k_mttkrp_flat<NOTHER, RR, RECB, true><<<grid, kWarps * 32, 0, st>>>(a); \
-    else k_mttkrp_flat<NOTHER, RR, RECB, false><<<grid, kWarps * 32, 0, st>>>(a);          \
-    return true;                                                                            \
-  }
-  FCASE(32) FCASE(64)
-#undef FCASE
-  return false;
-}
-
-// ---------------------------------------------------------------------------------
-// Asynchronous-gather variant (R = 32, short rows).
-// With factors far larger than L2 the plain kernel is bound by memory latency, not
-// bandwidth: a warp keeps only the gathers of ~1-2 steps in flight (registers), so
-// Delicious mode 2 moves 41 GB in 11.8 ms (3.5 TB/s).  Here the rows of the "big"
-// slots (bigmask: factors that stream from HBM) are copied by cp.async (LDGSTS, no
-// registers held) into a per-warp shared-memory ring 16-32 nonzeros ahead of the
-// products: the record batch of 32 nonzeros is split in two halves; while one half
-// is multiplied, the copies of the next half are in flight (cp.async.wait_group 1).
-// A half-warp copies one 256-byte row per instruction (16 lanes x 16 B, coalesced).
-// The arithmetic, its order and the row / carry logic are those of process_chunk
-// (G = 16 lanes per row, P = 2 nonzeros per step): results are bit-identical.
-constexpr int kAsyncWarps = 4;
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  const unsigned d = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(d), "l"(gmem));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
-__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;\n" ::); }
-
-template <int NOTHER, int RECB, bool HOT>
-__device__ __forceinline__ void process_chunk_async(const MArgs& a, int64_t c, const char* const* Fb,
-                                                    const char* const* HFb, int4* sr, double2* ring,
-                                                    int bigmask) {
-  constexpr int R = 32, RV = 16, G = 16, P = 2;
-  constexpr unsigned ROWB = R * 8;
-  constexpr int NW = RECB / 4;
-  constexpr int NV = RECB / 16;
-  const int lane = threadIdx.x & 31;
-  const int sg = lane / G, gl = lane % G;
-  int nbig = 0, bidx[NOTHER];
-#pragma unroll
-  for (int q = 0; q < NOTHER; q++) bidx[q] = ((bigmask >> q) & 1) ? nbig++ : -1;
-  // ring[slot t (0..31)][big slot b][RV double2]
-  const int64_t p0 = chunk_begin(a, c);
-  const int64_t p1 = chunk_end(a, c);
-  const int32_t ct = a.cont[c];
-  int64_t row = ct >= 0 ? (int64_t)ct : a.lb[c];
-  const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
-  double2 acc = make_double2(0.0, 0.0);
-  int64_t seg_end = (row < row_end) ? min(a.rowptr[row + 1], p1) : p1;
-  auto flush = [&](int64_t r) {
-    acc.x += __shfl_xor_sync(0xffffffffu, acc.x, 16);
-    acc.y += __shfl_xor_sync(0xffffffffu, acc.y, 16);
-    if (sg == 0) {
-      double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (r - a.rbase) * (int64_t)R;
-      reinterpret_cast<double2*>(dst)[gl] = acc;
-    }
-    acc = make_double2(0.0, 0.0);
-  };
-  // copies of the big-slot rows of 16 nonzeros: batch positions t0 .. t0+15 starting at
-  // nonzero pb0; the record of position t comes from `get(t, q)` (shared or registers)
-  auto issue = [&](int64_t pb0, int t0, auto get) {
-#pragma unroll
-    for (int i = 0; i < 8; i++) {
-      const int k = 2 * i + sg;                  // this half-warp's nonzero of the pair
-      const bool ok = pb0 + k < p1;
-#pragma unroll
-      for (int q = 0; q < NOTHER; q++) {
-        if (bidx[q] < 0) continue;
-        unsigned j = get(k, q);
-        const char* base = Fb[q];
-        if constexpr (HOT) {
-          if ((int)j < 0) { base = HFb[q]; j &= 0x7fffffffu; }
-        }
-        if (ok) cp_async16(ring + ((t0 + k) * nbig + bidx[q]) * RV + gl, row_addr<ROWB>(base, j));
-      }
-    }
-    cp_async_commit();
-  };
-  int4 nxt[NV];
-#pragma unroll
-  for (int k = 0; k < NV; k++)
-    nxt[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
-                              : make_int4(0, 0, 0, 0);
-  auto word_of = [](const int4& v, int w) { return (unsigned)(w == 0 ? v.x : w == 1 ? v.y : w == 2 ? v.z : v.w); };
-  auto from_sr = [&](int t) { return [=](int k, int q) { return word_of(sr[(t + k) * NV + q / 4], q % 4); }; };
-  // prologue: batch 0 published, its two halves in flight
-  __syncwarp();
-#pragma unroll
-  for (int k = 0; k < NV; k++) sr[lane * NV + k] = nxt[k];
-  __syncwarp();
-#pragma unroll
-  for (int k = 0; k < NV; k++)
-    nxt[k] = (p0 + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + 32 + lane) * RECB) + k)
-                                   : make_int4(0, 0, 0, 0);
-  issue(p0, 0, from_sr(0));
-  issue(p0 + 16, 16, from_sr(16));
-  for (int64_t pb = p0; pb < p1; pb += 32) {
-    const int nb = (int)min((int64_t)32, p1 - pb);
-    for (int half = 0; half < 2; half++) {
-      const int tlo = 16 * half, thi = min(16 * half + 16, nb);
-      cp_async_wait1();
-      __syncwarp();
-      int t = tlo;
-      while (t < thi) {
-        const int64_t p = pb + t;
-        if (p >= seg_end) {
-          flush(row);
-          row++;
-          seg_end = min(a.rowptr[row + 1], p1);
-          continue;
-        }
-        const int run = (int)min((int64_t)(thi - t), seg_end - p);
-#pragma unroll 4
-        for (int done = 0; done < run; done += P) {
-          const bool ok = (done + sg) < run;
-          const int src = ok ? t + done + sg : t + done;
-          unsigned w[NW];
-#pragma unroll
-          for (int k = 0; k < NV; k++) {
-            const int4 x = sr[src * NV + k];
-            w[4 * k] = x.x; w[4 * k + 1] = x.y; w[4 * k + 2] = x.z; w[4 * k + 3] = x.w;
-          }
-          const double v = ok ? __hiloint2double((int)w[NW - 1], (int)w[NW - 2]) : 0.0;
-          double2 f = make_double2(0.0, 0.0);
-#pragma unroll
-          for (int qq = 0; qq < NOTHER; qq++) {
-            double2 x;
-            if (bidx[qq] >= 0) {
-              x = ring[(src * nbig + bidx[qq]) * RV + gl];
-            } else {
-              const char* base = Fb[qq];
-              unsigned j = w[qq];
-              if constexpr (HOT) {
-                if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
-              }
-              x = *row_addr<ROWB>(base, j);
-            }
-            if (qq == 0) f = x;
-            else { f.x *= x.x; f.y *= x.y; }
-          }
-          acc.x = fma(v, f.x, acc.x);
-          acc.y = fma(v, f.y, acc.y);
-        }
-        t += run;
-      }
-      __syncwarp();            // every lane is done with this half's ring slots and records
-      if (half == 0) {         // next batch, first half: records still in registers
-        const int64_t pn = pb + 32;
-        issue(pn, 0, [&](int k, int q) { return (unsigned)__shfl_sync(0xffffffffu, (int)word_of(nxt[q / 4], q % 4), k); });
-      } else {                 // publish the next batch; its second half from shared memory
-#pragma unroll
-        for (int k = 0; k < NV; k++) sr[lane * NV + k] = nxt[k];
-        __syncwarp();
-#pragma unroll
-        for (int k = 0; k < NV; k++)
-          nxt[k] = (pb + 64 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 64 + lane) * RECB) + k)
-                                         : make_int4(0, 0, 0, 0);
-        issue(pb + 48, 16, from_sr(16));
-      }
-    }
-  }
-  asm volatile("cp.async.wait_all;\n" ::);
-  __syncwarp();
-  while (row < row_end) {
-    flush(row);
-    row++;
-  }
-}
-
-template <int NOTHER, int RECB, bool HOT>
-__global__ void __launch_bounds__(kAsyncWarps * 32, 3) k_mttkrp_async(MArgs a, int bigmask) {
-  extern __shared__ int4 dsm[];
-  constexpr int NV = RECB / 16;
-  const int warp = threadIdx.x >> 5, gl = (threadIdx.x & 31) % 16;
-  int nbig = 0;
-  for (int q = 0; q < NOTHER; q++) nbig += (bigmask >> q) & 1;
-  int4* sr = dsm + warp * 32 * NV;
-  double2* ring = reinterpret_cast<double2*>(dsm + kAsyncWarps * 32 * NV) + (size_t)warp * 32 * nbig * 16;
-  const char* Fb[NOTHER];
-  const char* HFb[NOTHER];
-#pragma unroll
-  for (int q = 0; q < NOTHER; q++) {
-    Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
-    HFb[q] = reinterpret_cast<const char*>(a.HF[q] ? a.HF[q] : a.F[q]) + gl * 16;
-  }
-  if (a.queue) {
-    for (;;) {
-      unsigned long long c = 0;
-      if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
-      c = __shfl_sync(0xffffffffu, c, 0);
-      if ((int64_t)c >= a.nchunks) break;
-      process_chunk_async<NOTHER, RECB, HOT>(a, (int64_t)c, Fb, HFb, sr, ring, bigmask);
-    }
-    return;
-  }
-  const int64_t nwarps = (int64_t)gridDim.x * kAsyncWarps;
-  for (int64_t c = blockIdx.x * (int64_t)kAsyncWarps + warp; c < a.nchunks; c += nwarps)
-    process_chunk_async<NOTHER, RECB, HOT>(a, c, Fb, HFb, sr, ring, bigmask);
-}
-
-size_t async_smem(int recb, int nbig) {
-  return (size_t)kAsyncWarps * 32 * recb + (size_t)kAsyncWarps * 32 * nbig * 256;
-}
-
-template <int NOTHER, int RECB>
-bool launch_async(const MArgs& a, int bigmask, bool hot, cudaStream_t st, int* grid_out) {
-  int nbig = 0;
-  for (int q = 0; q < NOTHER; q++) nbig += (bigmask >> q) & 1;
-  const size_t smem = async_smem(RECB, nbig);
-  static bool attr[2] = {false, false};
-  static int per_sm[2][8] = {{0}};
-  auto kern = hot ? k_mttkrp_async<NOTHER, RECB, true> : k_mttkrp_async<NOTHER, RECB, false>;
-  if (!attr[hot]) {
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)async_smem(RECB, NOTHER)) != cudaSuccess) { cudaGetLastError(); return false; }
-    attr[hot] = true;
-  }
-  if (!per_sm[hot][nbig]) {
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[hot][nbig], kern, kAsyncWarps * 32, smem) != cudaSuccess ||
-        per_sm[hot][nbig] < 1) { cudaGetLastError(); return false; }
-  }
-  const int64_t ctas = (a.nchunks + kAsyncWarps - 1) / kAsyncWarps;
-  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(ctas, (int64_t)device_info().sms * per_sm[hot][nbig]));
-  kern<<<grid, kAsyncWarps * 32, smem, st>>>(a, bigmask);
-  if (grid_out) *grid_out = grid;
-  return true;
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -858,35 +457,6 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, in
   const bool tl = a.ckb != nullptr;
   const int g = tl ? tgrid : grid;
   if (hot) gl = 0;                 // hot-row copies: the default group width (factors stream from HBM)
-  if (a.flat && !tl && (a.R == 32 || a.R == 64)) {
-    const int fg = std::min(grid, device_info().sms * 4);
-    switch (a.nother) {
-      case 2: done = launch_flat<2, 16>(a, hot, fg, st); break;
-      case 3: done = launch_flat<3, 32>(a, hot, fg, st); break;
-      case 4: done = launch_flat<4, 32>(a, hot, fg, st); break;
-      case 5: done = launch_flat<5, 32>(a, hot, fg, st); break;
-      case 6: done = launch_flat<6, 32>(a, hot, fg, st); break;
-      default: break;
-    }
-    if (done) {
-      CSTF_LAUNCHED();
-      return CSTF_OK;
-    }
-  }
-  if (a.async_mask && a.R == 32 && !tl) {
-    switch (a.nother) {
-      case 2: done = launch_async<2, 16>(a, a.async_mask, hot, st, nullptr); break;
-      case 3: done = launch_async<3, 32>(a, a.async_mask, hot, st, nullptr); break;
-      case 4: done = launch_async<4, 32>(a, a.async_mask, hot, st, nullptr); break;
-      case 5: done = launch_async<5, 32>(a, a.async_mask, hot, st, nullptr); break;
-      case 6: done = launch_async<6, 32>(a, a.async_mask, hot, st, nullptr); break;
-      default: break;
-    }
-    if (done) {
-      CSTF_LAUNCHED();
-      return CSTF_OK;
-    }
-  }
   switch (a.nother) {
     case 1: done = launch_fast<1, 16>(a, grid, st, false, gl, hot); break;
     case 2: done = launch_fast<2, 16>(a, g, st, tl, gl, hot); break;
@@ -1199,9 +769,6 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.wstart = nullptr;
   a.ckb = nullptr;
   a.queue = nullptr;
-  a.async_mask = 0;
-  a.pf_mask = 0;
-  a.flat = 0;
   a.pbase = 0;
   a.cbase = 0;
   a.rbase = 0;
@@ -1269,51 +836,6 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
     const char* ge = getenv("CSTF_MTTKRP_G");        // read per call (tests force both paths)
     if (ge && (atoi(ge) == 0 || atoi(ge) == 8)) gl = atoi(ge);
-  }
-  // Asynchronous gathers (k_mttkrp_async): R = 32, short rows (the 4-CTA/SM launches,
-  // latency-bound when factors stream from HBM), for the slots whose factor does not
-  // fit a quarter of L2.  Off by default (measured slower than the L2 prefetch below:
-  // DESIGN.md); CSTF_MTTKRP_ASYNC=1 enables it for short rows, =2 also for long rows,
-  // =3 forces every slot and every row length (tests at small sizes).
-  a.async_mask = 0;
-  {
-    const char* ae = getenv("CSTF_MTTKRP_ASYNC");
-    const int amode = ae ? atoi(ae) : 0;      // off by default: slower than the L2 prefetch
-    const bool short_rows = nnz < 64 * ms.Ivirt;
-    if (amode > 0 && R == 32 && N - 1 >= 2 && N - 1 <= 6 && !ms.slab && (short_rows || amode >= 2)) {
-      for (int q = 0; q < N - 1; q++) {
-        if (ms.tiled && q == ms.tslot && amode != 3) continue;   // the L2-blocked slot's slab is L2-resident
-        if (amode == 3 || X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) a.async_mask |= 1 << q;
-      }
-    }
-  }
-  // Flat stream (k_mttkrp_flat): R = 32 / 64 short-row copies that gather a factor
-  // larger than L2/4 (latency-bound).  CSTF_MTTKRP_FLAT=0 disables, =2 forces it
-  // for every R = 32 / 64 launch (tests).
-  {
-    const char* fe = getenv("CSTF_MTTKRP_FLAT");
-    const int fmode = fe ? atoi(fe) : 1;
-    const bool short_rows = nnz < 64 * ms.Ivirt;
-    bool big = false;
-    for (int q = 0; q < N - 1; q++)
-      if (!(ms.tiled && q == ms.tslot) && X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) big = true;
-    if ((R == 32 || R == 64) && N - 1 >= 2 && N - 1 <= 6 && !ms.slab && a.async_mask == 0 &&
-        ((fmode == 1 && short_rows && big) || fmode == 2))
-      a.flat = 1;
-  }
-  // L2 prefetch one record batch ahead for the slots whose factor does not fit a
-  // quarter of L2.  Off by default: measured slower (Delicious mode 0 9.4 -> 16 ms,
-  // DRAM reads 58 -> 108 GB: with ~4,700 warps each 32 nonzeros ahead, 77 MB of
-  // prefetched rows are in flight and evict each other before use).
-  // CSTF_MTTKRP_PF=1 enables it for those slots, =2 for every slot (tests).
-  {
-    const char* pe = getenv("CSTF_MTTKRP_PF");
-    const int pmode = pe ? atoi(pe) : 0;
-    if (pmode > 0 && !ms.slab && a.async_mask == 0)
-      for (int q = 0; q < N - 1; q++) {
-        if (ms.tiled && q == ms.tslot && pmode != 2) continue;
-        if (pmode == 2 || X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) a.pf_mask |= 1 << q;
-      }
   }
   int64_t nl = 0;
   if (ms.tiled && !ms.slab) {

@@ -731,81 +731,3 @@ def test_factorize_hot_row_tables(B, tol, R, monkeypatch):
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
     for a, b in zip(F, orc["factors"]):
         assert normwise(a, b) <= 1e-6
-
-
-@pytest.mark.parametrize("case", [("3mode", (300, 2111, 970), 200_000, (2, 2, 3)),
-                                  ("4mode", (90, 5000, 1200, 40), 200_000, (2, 2, 3, 1)),
-                                  ("2mode", (4000, 3000), 60_000, (2, 3)),
-                                  ("5mode", (30, 40, 50, 60, 20), 50_000, (2, 1, 2, 3, 1))])
-@pytest.mark.parametrize("hot", ["0", "150"])
-@pytest.mark.parametrize("knob", ["CSTF_MTTKRP_ASYNC=3", "CSTF_MTTKRP_PF=2", "CSTF_MTTKRP_FLAT=2"])
-def test_mttkrp_async_gathers(B, case, hot, knob, monkeypatch):
-    """k_mttkrp_async (cp.async row copies into a per-warp shared-memory ring, 16-32
-    nonzeros ahead of the products; R = 32) forced on every slot and mode
-    (CSTF_MTTKRP_ASYNC=3), with and without hot-row tables, against the oracle;
-    bitwise repeatable; rows without nonzeros stay zero.  The same checks for the
-    L2 bulk prefetch of the next record batch's rows forced on every slot, and for
-    the flat-stream kernel (one nonzero per warp step) forced on every launch."""
-    k, v = knob.split("=")
-    monkeypatch.setenv(k, v)
-    if hot != "0":
-        monkeypatch.setenv("CSTF_HOT_ROWS", hot)
-    else:
-        monkeypatch.setenv("CSTF_HOT", "0")
-    name, dims, nnz, gam = case
-    idx, vals = datagen.coo(dims, gam, nnz, 61)
-    idx[0] = (idx[0] // 2 * 2).astype(np.int32)                 # odd rows of mode 0 empty
-    X = B.cstf_tensor_load_coo(dims, idx, vals)
-    ref = oracle.coalesce(dims, idx, vals)
-    F = datagen.init_factors(dims, 32, 12)
-    Fd = [cu(f) for f in F]
-    for n in range(len(dims)):
-        M = cu(np.full((dims[n], 32), np.nan))
-        B.cstf_mttkrp(X, n, Fd, M)
-        got = host(M).copy()
-        assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, (name, n)
-        B.cstf_mttkrp(X, n, Fd, M)
-        assert np.array_equal(host(M), got), (name, n)
-        if n == 0:
-            assert np.all(got[1::2] == 0.0)
-
-
-@pytest.mark.parametrize("knob", ["CSTF_MTTKRP_ASYNC=3", "CSTF_MTTKRP_FLAT=2"])
-def test_factorize_async_gathers(B, knob, monkeypatch):
-    """The factorisation with asynchronous gathers / the flat stream forced (and hot
-    rows) vs the oracle."""
-    k, v = knob.split("=")
-    monkeypatch.setenv(k, v)
-    monkeypatch.setenv("CSTF_HOT_ROWS", "200")
-    c = datagen.CONFIGS["delicious"].scaled(1000, nnz_factor=700)
-    idx, vals = c.generate()
-    start = datagen.init_factors(c.dims, 32, c.seed)
-    orc, gpu, F, lam = run_both(B, c.dims, idx, vals, 32, start, outer=4, tol=1e-2)
-    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
-    assert tie is None
-    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
-    for a, b in zip(F, orc["factors"]):
-        assert normwise(a, b) <= 1e-6
-
-
-@pytest.mark.parametrize("R", [32, 64])
-def test_mttkrp_flat_window_slides(B, R, monkeypatch):
-    """Flat stream: a chunk crossing > 32 rows inside one record batch (runs of empty
-    rows between single-nonzero rows) slides the 32-row window; heavy rows split over
-    chunks go through the carry fix-up."""
-    monkeypatch.setenv("CSTF_MTTKRP_FLAT", "2")
-    rng = np.random.default_rng(R)
-    nnz = 120_000
-    I = 200_000
-    i = rng.integers(0, I, nnz).astype(np.int32)          # ~0.6 nonzeros per row: long empty runs
-    i[:30_000] = 17                                        # one heavy row over many chunks
-    dims = (I, 700, 300)
-    j = rng.integers(0, 700, nnz).astype(np.int32)
-    k = rng.integers(0, 300, nnz).astype(np.int32)
-    vals = rng.random(nnz)
-    X = B.cstf_tensor_load_coo(dims, [i, j, k], vals)
-    ref = oracle.coalesce(dims, [i, j, k], vals)
-    F = [rng.random((d, R)) for d in dims]
-    M = cu(np.full((I, R), np.nan))
-    B.cstf_mttkrp(X, 0, [cu(f) for f in F], M)
-    assert normwise(host(M), oracle.mttkrp(ref, 0, F)) <= TOL

@@ -146,14 +146,17 @@ __device__ __forceinline__ void acc4(double h, double ht, double h0, double u, d
   r += e1 * e1; s += e2 * e2; nh += h * h; nu += u * u;
 }
 // residual sums of the baseline (the norms of Alg. 2 l.9, one pass over the four matrices)
+// (explicit loops: accumulators captured by reference in a lambda went to local memory)
 __global__ void k_resid(const double* __restrict__ H, const double* __restrict__ Ht, const double* __restrict__ H0,
                         const double* __restrict__ U, int64_t n, double* __restrict__ part) {
   double r = 0, s = 0, h = 0, u = 0;
-  elemwise(n, [&](int64_t x) {
+  const int64_t n2 = n >> 1;
+  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n2; x += (int64_t)gridDim.x * kT) {
     const double2 a = ld2(H, x), t = ld2(Ht, x), z = ld2(H0, x), v = ld2(U, x);
     acc4(a.x, t.x, z.x, v.x, r, s, h, u);
     acc4(a.y, t.y, z.y, v.y, r, s, h, u);
-  }, [&](int64_t x) { acc4(H[x], Ht[x], H0[x], U[x], r, s, h, u); });
+  }
+  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) acc4(H[n - 1], Ht[n - 1], H0[n - 1], U[n - 1], r, s, h, u);
   block_store4(r, s, h, u, part);
 }
 
@@ -177,19 +180,21 @@ __device__ __forceinline__ void epi1(double ht, double h0, double u0, double& hn
 __global__ void k_fused_epi(const double* __restrict__ Ht, double* __restrict__ H, double* __restrict__ U, int64_t n,
                             double* __restrict__ part) {
   double r = 0, s = 0, h = 0, u = 0;
-  elemwise(n, [&](int64_t x) {
+  const int64_t n2 = n >> 1;
+  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n2; x += (int64_t)gridDim.x * kT) {
     const double2 t = ld2(Ht, x), h0 = ld2(H, x), u0 = ld2(U, x);
     double a, b, c, d;
     epi1(t.x, h0.x, u0.x, a, c, r, s, h, u);
     epi1(t.y, h0.y, u0.y, b, d, r, s, h, u);
     st2(H, x, a, b);
     st2(U, x, c, d);
-  }, [&](int64_t x) {
+  }
+  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) {
     double a, c;
-    epi1(Ht[x], H[x], U[x], a, c, r, s, h, u);
-    H[x] = a;
-    U[x] = c;
-  });
+    epi1(Ht[n - 1], H[n - 1], U[n - 1], a, c, r, s, h, u);
+    H[n - 1] = a;
+    U[n - 1] = c;
+  }
   block_store4(r, s, h, u, part);
 }
 

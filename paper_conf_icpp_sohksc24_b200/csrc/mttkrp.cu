@@ -117,15 +117,6 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
 #pragma unroll
     for (int s = 0; s < VPL; s++) acc[s] = make_double2(0.0, 0.0);
     int64_t seg_end = (row < row_end) ? min(a.rowptr[row + 1], p1) : p1;
-    // Row-end window: lane L holds rowptr[wrow + 1 + L], so the next row's end comes
-    // from a shuffle instead of a dependent load per row (short rows: one load per 32
-    // rows).  Indices past the chunk's rows read as "beyond p1".
-    int64_t wrow = row;
-    auto load_window = [&]() {
-      const int64_t r = wrow + 1 + lane;
-      return (r < row_end) ? a.rowptr[r] : INT64_MAX;
-    };
-    int64_t wend = load_window();
 
     auto flush = [&](int64_t r) {
 #pragma unroll
@@ -170,11 +161,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
         if (p >= seg_end) {
           flush(row);
           row++;
-          if (row - wrow >= 32) {
-            wrow = row;
-            wend = load_window();
-          }
-          seg_end = min(__shfl_sync(0xffffffffu, wend, (int)(row - wrow)), p1);
+          seg_end = min(a.rowptr[row + 1], p1);
           continue;
         }
         const int run = (int)min((int64_t)(nb - t), seg_end - p);

@@ -10,6 +10,7 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <functional>
 #include <cstdlib>
 #include <cstring>
 #include <vector>
@@ -353,14 +354,22 @@ cstf_status build_rowptr(const int32_t* d_key, int64_t n, int64_t I, DevBuf& row
 //     (Amazon: 678 -> ~569 ms of MTTKRP per outer iteration).
 //  Delicious modes 1-3 satisfy neither (blocking them measured slower).
 //  CSTF_L2_BLOCK_ROWS / CSTF_L2_BLOCK_MAXROWS force it (tests, experiments).
-void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int64_t* Ioth) {
+// cov (optional, single GPU): per slot, the share of the nonzeros that fall on the
+// factor's L2-capacity hottest rows (decide_hot).  When several other factors
+// qualify, the one with the FLATTEST distribution (lowest share) is blocked and the
+// skewed ones stream, since their hot rows are the ones a cache keeps (reading of
+// VERDICT r01 "skew-aware blocking"; CSTF_L2_BLOCK_SKEW=0: always the longest).
+void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int64_t* Ioth,
+                     const double* cov = nullptr) {
   if (N < 3 || (getenv("CSTF_L2_BLOCK") && atoi(getenv("CSTF_L2_BLOCK")) == 0)) return;
   const char* ov = getenv("CSTF_L2_BLOCK_ROWS");
   const bool forced = ov != nullptr;
   const int64_t l2rows = ov && atoll(ov) > 0 ? atoll(ov) : kL2Rows;
   const int64_t maxv = getenv("CSTF_L2_BLOCK_MAXROWS") ? atoll(getenv("CSTF_L2_BLOCK_MAXROWS"))
                                                       : ((int64_t)16 << 20);
-  for (int q = N - 2; q >= (forced ? 0 : N - 2) && !ms.tiled; q--) {     // largest other factor first
+  const bool skew = cov && !forced && !(getenv("CSTF_L2_BLOCK_SKEW") && atoi(getenv("CSTF_L2_BLOCK_SKEW")) == 0);
+  int best = -1;
+  for (int q = N - 2; q >= ((forced || skew) ? 0 : N - 2); q--) {     // largest other factor first
     const int64_t It = Ioth[q];
     const int64_t nb = (It + l2rows - 1) / l2rows;
     bool ok = It > 2 * l2rows && nb * Iloc < ((int64_t)1 << 31) && nloc >= 4 * nb * Iloc;
@@ -368,9 +377,13 @@ void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int
       ok = ok && nb * Iloc <= maxv;
     else
       ok = ok && It * 256 > (int64_t)device_info().l2 && (nb * Iloc * 64 <= nloc || nloc >= 8 * nb * Iloc);
-    if (ok) {
-      ms.tiled = true; ms.slab = false; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = q;
-    }
+    if (!ok) continue;
+    if (!skew) { best = q; break; }
+    if (best < 0 || cov[q] < cov[best]) best = q;
+  }
+  if (best >= 0) {
+    const int64_t nb = (Ioth[best] + l2rows - 1) / l2rows;
+    ms.tiled = true; ms.slab = false; ms.blk_rows = l2rows; ms.nblk = nb; ms.tslot = best;
   }
 }
 
@@ -521,16 +534,20 @@ cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int
 // descending count order.  CSTF_HOT=0 disables; CSTF_HOT_ROWS=<n> forces n hot rows
 // per factor that has more than 2n rows (tests).  hmap[k] (device int32[I_k]) maps a
 // row to its hot slot or -1 and is used while the mode copies are built.
-cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap, cudaStream_t st) {
+// Also fills cov[k] (all factors larger than half the L2 at R = 32): the share of the
+// nonzeros on the factor's L2-capacity hottest rows, for the skew-aware L2-block choice.
+cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap, double* cov, cudaStream_t st) {
   const int N = X->N;
   X->hot_total = 0;
-  if (N < 3 || (getenv("CSTF_HOT") && atoi(getenv("CSTF_HOT")) == 0)) return CSTF_OK;
+  for (int k = 0; k < N; k++) cov[k] = 1.0;
+  if (N < 3) return CSTF_OK;
+  const bool hot_on = !(getenv("CSTF_HOT") && atoi(getenv("CSTF_HOT")) == 0);
   const char* fe = getenv("CSTF_HOT_ROWS");
   const int64_t forced = fe ? atoll(fe) : 0;
   int maxp = 0;
   cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, device_info().device);
-  const int64_t per_factor = forced > 0 ? forced : (int64_t)maxp / 256 / 2;
-  if (per_factor < 1) return CSTF_OK;
+  const int64_t per_factor = !hot_on ? 0 : forced > 0 ? forced : (int64_t)maxp / 256 / 2;
+  const int64_t l2rows = (int64_t)device_info().l2 / 256;
   std::vector<int32_t> all;
   for (int k = 0; k < N; k++) {
     X->hot_off[k] = (int64_t)all.size();
@@ -550,6 +567,15 @@ cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap
     for (int64_t i = 0; i < I; i++) order[(size_t)i] = (int32_t)i;
     const int64_t H = std::min<int64_t>(per_factor, I);
     auto by_count = [&](int32_t a, int32_t b) { return counts[a] != counts[b] ? counts[a] > counts[b] : a < b; };
+    {
+      std::vector<int64_t> cs(counts);
+      const int64_t C = std::min<int64_t>(l2rows, I);
+      std::nth_element(cs.begin(), cs.begin() + (C - 1), cs.end(), std::greater<int64_t>());
+      double top = 0.0;
+      for (int64_t i = 0; i < C; i++) top += (double)cs[(size_t)i];
+      cov[k] = top / (double)nout;
+    }
+    if (H < 1) continue;
     std::partial_sort(order.begin(), order.begin() + H, order.end(), by_count);
     int64_t h = 0;
     while (h < H && counts[(size_t)order[(size_t)h]] >= 2) h++;
@@ -679,8 +705,10 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
   if (X->partitioned) return build_partitioned(X, c_idx, c_vals, nout, tmp, st);
   // ---- 6. hot rows of the factors much larger than L2 (single GPU)
   DevBuf hmap[8];
+  double cov[8];
   static const bool kblock_env = getenv("CSTF_KBLOCK") && atoi(getenv("CSTF_KBLOCK")) > 0;
-  if (!kblock_env) CSTF_TRY(decide_hot(X, c_idx, nout, hmap, st));
+  for (int k = 0; k < 8; k++) cov[k] = 1.0;
+  if (!kblock_env) CSTF_TRY(decide_hot(X, c_idx, nout, hmap, cov, st));
   // ---- 7. per-mode copies: sorted by (i_n, other modes by increasing length), AoS records
   const int recb = record_bytes(N);
   for (int n_ = 0; n_ < N; n_++) {
@@ -712,8 +740,9 @@ cstf_status build_store(cstf_tensor* X, const int32_t* const* host_idx, const do
       }
     } else {
       int64_t Ioth[7];
-      for (int q = 0; q < N - 1; q++) Ioth[q] = X->dims[ms.other[q]];
-      decide_l2_block(ms, N, nout, ms.I, Ioth);
+      double cq[7];
+      for (int q = 0; q < N - 1; q++) { Ioth[q] = X->dims[ms.other[q]]; cq[q] = cov[ms.other[q]]; }
+      decide_l2_block(ms, N, nout, ms.I, Ioth, cq);
       if (ms.tiled) t = ms.other[ms.tslot];
     }
     const int64_t nblk = ms.nblk;

@@ -369,6 +369,8 @@ void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int
                                                       : ((int64_t)16 << 20);
   const bool skew = cov && !forced && !(getenv("CSTF_L2_BLOCK_SKEW") && atoi(getenv("CSTF_L2_BLOCK_SKEW")) == 0);
   int best = -1;
+  // the longest other factor decides WHETHER the copy is blocked; with `skew`, a
+  // flatter qualifying factor may then be blocked in its place
   for (int q = N - 2; q >= ((forced || skew) ? 0 : N - 2); q--) {     // largest other factor first
     const int64_t It = Ioth[q];
     const int64_t nb = (It + l2rows - 1) / l2rows;
@@ -377,7 +379,10 @@ void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int
       ok = ok && nb * Iloc <= maxv;
     else
       ok = ok && It * 256 > (int64_t)device_info().l2 && (nb * Iloc * 64 <= nloc || nloc >= 8 * nb * Iloc);
-    if (!ok) continue;
+    if (!ok) {
+      if (skew && q == N - 2) break;        // the longest does not qualify: not blocked
+      continue;
+    }
     if (!skew) { best = q; break; }
     if (best < 0 || cov[q] < cov[best]) best = q;
   }

@@ -46,7 +46,6 @@ struct MArgs {
   double* carry;        // [nchunks][R]
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
-  int bulk_mask;        // != 0: k_mttkrp_bulk; slots whose rows arrive by TMA bulk copies (R = 32)
 };
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
@@ -240,260 +239,6 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
     return;
   }
   for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT>(a, c, Fb, srec, HFb);
-}
-
-// ---------------------------------------------------------------------------------
-// TMA bulk-copy variant (R = 32).  Short-row
-// copies of factors far larger than L2 are bound by memory latency: a warp of the
-// plain kernel has the gathers of 1-2 steps in flight in registers.  Here the rows of
-// the "big" slots (bulk_mask) are fetched by the TMA engine, cp.async.bulk of one
-// whole 256-byte row per instruction, issued by the lane that holds the nonzero's
-// record, into a per-warp ring of 2 quarters x 8 nonzeros in shared memory with one
-// mbarrier per quarter slot (complete_tx); quarter g + 2 is requested as soon as
-// quarter g has been multiplied.  No registers are held by the loads and the copy
-// costs 1 instruction per row instead of 16 lanes x 16 B.  Product order and row /
-// carry logic as in process_chunk (runs split at quarter boundaries).
-constexpr int kBulkQ = 8;       // nonzeros per quarter
-
-__device__ __forceinline__ void mbar_init(uint64_t* mb) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"((unsigned)__cvta_generic_to_shared(mb)));
-}
-__device__ __forceinline__ void mbar_expect(uint64_t* mb, unsigned bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"((unsigned)__cvta_generic_to_shared(mb)),
-               "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* mb, unsigned parity) {
-  const unsigned a = (unsigned)__cvta_generic_to_shared(mb);
-  unsigned done = 0;
-  do {
-    asm volatile("{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-                 : "=r"(done) : "r"(a), "r"(parity) : "memory");
-  } while (!done);
-}
-__device__ __forceinline__ void bulk_row(void* dst, const void* src, uint64_t* mb) {
-  asm volatile("cp.async.bulk.shared::cta.global.mbarrier::complete_tx::bytes [%0], [%1], 256, [%2];\n" ::
-                   "r"((unsigned)__cvta_generic_to_shared(dst)), "l"(src), "r"((unsigned)__cvta_generic_to_shared(mb))
-               : "memory");
-}
-
-template <int NOTHER, int RECB, bool HOT>
-__device__ __forceinline__ void process_chunk_bulk(const MArgs& a, int64_t c, const char* const* Fb,
-                                                   const char* const* HFb, int4* sr, double2* ring, uint64_t* mb,
-                                                   unsigned& ph, int nbig, const int* bidx) {
-  constexpr int R = 32, RV = 16, G = 16, P = 2;
-  constexpr unsigned ROWB = R * 8;
-  constexpr int NW = RECB / 4;
-  constexpr int NV = RECB / 16;
-  const int lane = threadIdx.x & 31;
-  const int sg = lane / G, gl = lane % G;
-  const int64_t p0 = chunk_begin(a, c);
-  const int64_t p1 = chunk_end(a, c);
-  const int32_t ct = a.cont[c];
-  int64_t row = ct >= 0 ? (int64_t)ct : a.lb[c];
-  const int64_t row_end = (c == a.nchunks - 1) ? a.I : a.lb[c + 1];
-  double2 acc = make_double2(0.0, 0.0);
-  int64_t seg_end = (row < row_end) ? min(a.rowptr[row + 1], p1) : p1;
-  auto flush = [&](int64_t r) {
-    acc.x += __shfl_xor_sync(0xffffffffu, acc.x, 16);
-    acc.y += __shfl_xor_sync(0xffffffffu, acc.y, 16);
-    if (sg == 0) {
-      double* dst = (ct >= 0 && r == (int64_t)ct) ? a.carry + c * (int64_t)R : a.M + (r - a.rbase) * (int64_t)R;
-      reinterpret_cast<double2*>(dst)[gl] = acc;
-    }
-    acc = make_double2(0.0, 0.0);
-  };
-  // request quarter g (nonzeros pq .. pq+7) into slot g & 1; lane 8k+L of the batch owns
-  // the record of position 8k+L, so lanes [8 (g%4), 8 (g%4) + 8) issue the copies
-  auto request = [&](int64_t pq, int g, const int4 (&rec)[NV]) {
-    const int slot = g & 1;
-    const int qk = g & 3;
-    const int64_t nvalid = max((int64_t)0, min((int64_t)kBulkQ, p1 - pq));
-    // the slot's previous contents were read through the generic proxy: order those
-    // reads before the async-proxy (TMA) writes into it
-    asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-    if (lane == 0) mbar_expect(mb + slot, (unsigned)(nvalid * nbig * 256));
-    __syncwarp();
-    const int L = lane - kBulkQ * qk;
-    if (L >= 0 && L < nvalid) {
-#pragma unroll
-      for (int q = 0; q < NOTHER; q++) {
-        if (bidx[q] < 0) continue;
-        const int4 v = rec[q / 4];
-        unsigned j = (unsigned)((q % 4) == 0 ? v.x : (q % 4) == 1 ? v.y : (q % 4) == 2 ? v.z : v.w);
-        const char* base = Fb[q] - gl * 16;
-        if constexpr (HOT) {
-          if ((int)j < 0) { base = HFb[q] - gl * 16; j &= 0x7fffffffu; }
-        }
-        bulk_row(ring + ((slot * kBulkQ + L) * nbig + bidx[q]) * RV, row_addr<ROWB>(base, j), mb + slot);
-      }
-    }
-  };
-  int4 cur[NV], nxt[NV];
-#pragma unroll
-  for (int k = 0; k < NV; k++)
-    cur[k] = (p0 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + lane) * RECB) + k)
-                              : make_int4(0, 0, 0, 0);
-#pragma unroll
-  for (int k = 0; k < NV; k++)
-    nxt[k] = (p0 + 32 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (p0 + 32 + lane) * RECB) + k)
-                                   : make_int4(0, 0, 0, 0);
-  __syncwarp();
-#pragma unroll
-  for (int k = 0; k < NV; k++) sr[lane * NV + k] = cur[k];
-  request(p0, 0, cur);
-  request(p0 + kBulkQ, 1, cur);
-  int g = 0;                                         // quarter being multiplied (chunk-relative)
-  for (int64_t pb = p0; pb < p1; pb += 32) {
-    const int nb = (int)min((int64_t)32, p1 - pb);
-    for (int qk = 0; qk < 4; qk++, g++) {
-      const int tlo = kBulkQ * qk;
-      const int thi = min(tlo + kBulkQ, nb);
-      const int slot = g & 1;
-      mbar_wait(mb + slot, (ph >> slot) & 1);
-      ph ^= 1u << slot;
-      if (tlo < thi) {
-        int t = tlo;
-        while (t < thi) {
-          const int64_t p = pb + t;
-          if (p >= seg_end) {
-            flush(row);
-            row++;
-            seg_end = min(a.rowptr[row + 1], p1);
-            continue;
-          }
-          const int run = (int)min((int64_t)(thi - t), seg_end - p);
-#pragma unroll 4
-          for (int done = 0; done < run; done += P) {
-            const bool ok = (done + sg) < run;
-            const int src = ok ? t + done + sg : t + done;
-            unsigned w[NW];
-#pragma unroll
-            for (int k = 0; k < NV; k++) {
-              const int4 x = sr[src * NV + k];
-              w[4 * k] = x.x; w[4 * k + 1] = x.y; w[4 * k + 2] = x.z; w[4 * k + 3] = x.w;
-            }
-            const double v = ok ? __hiloint2double((int)w[NW - 1], (int)w[NW - 2]) : 0.0;
-            double2 f = make_double2(0.0, 0.0);
-#pragma unroll
-            for (int qq = 0; qq < NOTHER; qq++) {
-              double2 x;
-              if (bidx[qq] >= 0) {
-                x = ring[((slot * kBulkQ + (src - tlo)) * nbig + bidx[qq]) * RV + gl];
-              } else {
-                const char* base = Fb[qq];
-                unsigned j = w[qq];
-                if constexpr (HOT) {
-                  if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
-                }
-                x = *row_addr<ROWB>(base, j);
-              }
-              if (qq == 0) f = x;
-              else { f.x *= x.x; f.y *= x.y; }
-            }
-            acc.x = fma(v, f.x, acc.x);
-            acc.y = fma(v, f.y, acc.y);
-          }
-          t += run;
-        }
-      }
-      __syncwarp();                                  // slot g & 1 is free again
-      const int gn = g + 2;                          // request quarter g + 2
-      if (qk < 2) {
-        request(pb + kBulkQ * (qk + 2), gn, cur);
-      } else {
-        request(pb + 32 + kBulkQ * (qk - 2), gn, nxt);
-      }
-    }
-    // next batch: its records become current (shared memory), the one after is loaded
-#pragma unroll
-    for (int k = 0; k < NV; k++) cur[k] = nxt[k];
-#pragma unroll
-    for (int k = 0; k < NV; k++)
-      nxt[k] = (pb + 64 + lane < p1) ? __ldcs(reinterpret_cast<const int4*>(a.rec + (pb + 64 + lane) * RECB) + k)
-                                     : make_int4(0, 0, 0, 0);
-    __syncwarp();
-#pragma unroll
-    for (int k = 0; k < NV; k++) sr[lane * NV + k] = cur[k];
-    __syncwarp();
-  }
-  // the two requests past the end (empty or partial): consume their phases
-  for (int k = 0; k < 2; k++, g++) {
-    const int slot = g & 1;
-    mbar_wait(mb + slot, (ph >> slot) & 1);
-    ph ^= 1u << slot;
-  }
-  __syncwarp();
-  while (row < row_end) {
-    flush(row);
-    row++;
-  }
-}
-
-template <int NOTHER, int RECB, bool HOT>
-__global__ void __launch_bounds__(kWarps * 32, 3) k_mttkrp_bulk(MArgs a) {
-  extern __shared__ __align__(128) unsigned char bsm[];
-  constexpr int NV = RECB / 16;
-  const int warp = threadIdx.x >> 5, gl = (threadIdx.x & 31) % 16;
-  int nbig = 0, bidx[NOTHER];
-#pragma unroll
-  for (int q = 0; q < NOTHER; q++) bidx[q] = ((a.bulk_mask >> q) & 1) ? nbig++ : -1;
-  uint64_t* mb = reinterpret_cast<uint64_t*>(bsm) + warp * 2;                      // [warp][2]
-  int4* sr = reinterpret_cast<int4*>(bsm + kWarps * 2 * 8) + warp * 32 * NV;        // [warp][32][NV]
-  double2* ring = reinterpret_cast<double2*>(bsm + kWarps * 2 * 8 + kWarps * 32 * RECB) +
-                  (size_t)warp * 2 * kBulkQ * nbig * 16;                          // [warp][2][8][nbig][16]
-  if ((threadIdx.x & 31) == 0) {
-    mbar_init(mb);
-    mbar_init(mb + 1);
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
-  __syncwarp();
-  unsigned ph = 0;
-  const char* Fb[NOTHER];
-  const char* HFb[NOTHER];
-#pragma unroll
-  for (int q = 0; q < NOTHER; q++) {
-    Fb[q] = reinterpret_cast<const char*>(a.F[q]) + gl * 16;
-    HFb[q] = reinterpret_cast<const char*>(a.HF[q] ? a.HF[q] : a.F[q]) + gl * 16;
-  }
-  if (a.queue) {
-    for (;;) {
-      unsigned long long c = 0;
-      if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
-      c = __shfl_sync(0xffffffffu, c, 0);
-      if ((int64_t)c >= a.nchunks) break;
-      process_chunk_bulk<NOTHER, RECB, HOT>(a, (int64_t)c, Fb, HFb, sr, ring, mb, ph, nbig, bidx);
-    }
-    return;
-  }
-  const int64_t nwarps = (int64_t)gridDim.x * kWarps;
-  for (int64_t c = blockIdx.x * (int64_t)kWarps + warp; c < a.nchunks; c += nwarps)
-    process_chunk_bulk<NOTHER, RECB, HOT>(a, c, Fb, HFb, sr, ring, mb, ph, nbig, bidx);
-}
-
-size_t bulk_smem(int recb, int nbig) {
-  return (size_t)kWarps * 2 * 8 + (size_t)kWarps * 32 * recb + (size_t)kWarps * 2 * kBulkQ * nbig * 256;
-}
-
-template <int NOTHER, int RECB>
-bool launch_bulk(const MArgs& a, bool hot, int grid, cudaStream_t st) {
-  int nbig = 0;
-  for (int q = 0; q < NOTHER; q++) nbig += (a.bulk_mask >> q) & 1;
-  const size_t smem = bulk_smem(RECB, nbig);
-  auto kern = hot ? k_mttkrp_bulk<NOTHER, RECB, true> : k_mttkrp_bulk<NOTHER, RECB, false>;
-  static bool attr[2] = {false, false};
-  static int per_sm[2][8] = {{0}};
-  if (!attr[hot]) {
-    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bulk_smem(RECB, NOTHER)) !=
-        cudaSuccess) { cudaGetLastError(); return false; }
-    attr[hot] = true;
-  }
-  if (!per_sm[hot][nbig]) {
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm[hot][nbig], kern, kWarps * 32, smem) != cudaSuccess ||
-        per_sm[hot][nbig] < 1) { cudaGetLastError(); return false; }
-  }
-  grid = (int)std::max(1, std::min(grid, device_info().sms * per_sm[hot][nbig]));
-  kern<<<grid, kWarps * 32, smem, st>>>(a);
-  return true;
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -712,21 +457,6 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, in
   const bool tl = a.ckb != nullptr;
   const int g = tl ? tgrid : grid;
   if (hot) gl = 0;                 // hot-row copies: the default group width (factors stream from HBM)
-  if (a.bulk_mask && a.R == 32 && !tl) {
-    const int bg = (int)std::min<int64_t>((a.nchunks + kWarps - 1) / kWarps, (int64_t)device_info().sms * 8);
-    switch (a.nother) {
-      case 2: done = launch_bulk<2, 16>(a, hot, bg, st); break;
-      case 3: done = launch_bulk<3, 32>(a, hot, bg, st); break;
-      case 4: done = launch_bulk<4, 32>(a, hot, bg, st); break;
-      case 5: done = launch_bulk<5, 32>(a, hot, bg, st); break;
-      case 6: done = launch_bulk<6, 32>(a, hot, bg, st); break;
-      default: break;
-    }
-    if (done) {
-      CSTF_LAUNCHED();
-      return CSTF_OK;
-    }
-  }
   switch (a.nother) {
     case 1: done = launch_fast<1, 16>(a, grid, st, false, gl, hot); break;
     case 2: done = launch_fast<2, 16>(a, g, st, tl, gl, hot); break;
@@ -1039,7 +769,6 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.wstart = nullptr;
   a.ckb = nullptr;
   a.queue = nullptr;
-  a.bulk_mask = 0;
   a.pbase = 0;
   a.cbase = 0;
   a.rbase = 0;
@@ -1107,19 +836,6 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
     if (R == 32 && gbytes <= (int64_t)di.l2) gl = 8;
     const char* ge = getenv("CSTF_MTTKRP_G");        // read per call (tests force both paths)
     if (ge && (atoi(ge) == 0 || atoi(ge) == 8)) gl = atoi(ge);
-  }
-  // TMA bulk-copy gathers (k_mttkrp_bulk): R = 32 short-row copies, for the slots whose
-  // factor does not fit a quarter of L2.  CSTF_MTTKRP_BULK=0 disables, =2 also long
-  // rows, =3 forces every slot of every launch (tests).
-  {
-    const char* be = getenv("CSTF_MTTKRP_BULK");
-    const int bmode = be ? atoi(be) : 0;
-    const bool short_rows = nnz < 64 * ms.Ivirt;
-    if (bmode > 0 && R == 32 && N - 1 >= 2 && N - 1 <= 6 && !ms.slab && (short_rows || bmode >= 2))
-      for (int q = 0; q < N - 1; q++) {
-        if (ms.tiled && q == ms.tslot && bmode != 3) continue;
-        if (bmode == 3 || X->dims[ms.other[q]] * (int64_t)R * 8 > (int64_t)di.l2 / 4) a.bulk_mask |= 1 << q;
-      }
   }
   int64_t nl = 0;
   if (ms.tiled && !ms.slab) {

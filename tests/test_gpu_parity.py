@@ -731,49 +731,3 @@ def test_factorize_hot_row_tables(B, tol, R, monkeypatch):
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
     for a, b in zip(F, orc["factors"]):
         assert normwise(a, b) <= 1e-6
-
-
-@pytest.mark.parametrize("case", [("3mode", (300, 2111, 970), 200_000, (2, 2, 3)),
-                                  ("4mode", (90, 5000, 1200, 40), 200_000, (2, 2, 3, 1)),
-                                  ("5mode", (30, 40, 50, 60, 20), 50_000, (2, 1, 2, 3, 1))])
-@pytest.mark.parametrize("hot", ["0", "150"])
-def test_mttkrp_bulk_copy_gathers(B, case, hot, monkeypatch):
-    """k_mttkrp_bulk (TMA cp.async.bulk row copies into a per-warp shared-memory ring,
-    mbarrier completion; R = 32) forced on every slot and launch (CSTF_MTTKRP_BULK=3),
-    with and without hot-row tables: every mode against the oracle, bitwise
-    repeatable, rows without nonzeros zero."""
-    monkeypatch.setenv("CSTF_MTTKRP_BULK", "3")
-    if hot != "0":
-        monkeypatch.setenv("CSTF_HOT_ROWS", hot)
-    else:
-        monkeypatch.setenv("CSTF_HOT", "0")
-    name, dims, nnz, gam = case
-    idx, vals = datagen.coo(dims, gam, nnz, 61)
-    idx[0] = (idx[0] // 2 * 2).astype(np.int32)                 # odd rows of mode 0 empty
-    X = B.cstf_tensor_load_coo(dims, idx, vals)
-    ref = oracle.coalesce(dims, idx, vals)
-    F = datagen.init_factors(dims, 32, 12)
-    Fd = [cu(f) for f in F]
-    for n in range(len(dims)):
-        M = cu(np.full((dims[n], 32), np.nan))
-        B.cstf_mttkrp(X, n, Fd, M)
-        got = host(M).copy()
-        assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, (name, n)
-        B.cstf_mttkrp(X, n, Fd, M)
-        assert np.array_equal(host(M), got), (name, n)
-        if n == 0:
-            assert np.all(got[1::2] == 0.0)
-
-
-def test_factorize_bulk_copy_gathers(B, monkeypatch):
-    monkeypatch.setenv("CSTF_MTTKRP_BULK", "3")
-    monkeypatch.setenv("CSTF_HOT_ROWS", "200")
-    c = datagen.CONFIGS["delicious"].scaled(1000, nnz_factor=700)
-    idx, vals = c.generate()
-    start = datagen.init_factors(c.dims, 32, c.seed)
-    orc, gpu, F, lam = run_both(B, c.dims, idx, vals, 32, start, outer=4, tol=1e-2)
-    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
-    assert tie is None
-    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
-    for a, b in zip(F, orc["factors"]):
-        assert normwise(a, b) <= 1e-6

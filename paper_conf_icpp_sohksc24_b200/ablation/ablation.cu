@@ -101,32 +101,41 @@ __global__ void k_chol(const double* __restrict__ S, int R, int want_inv, double
 }
 
 // Element-wise kernels: 16-byte (double2) accesses over the flat I x R array, grid
-// = 16 CTAs per SM (enough 16-byte loads in flight to stream at HBM rate); an odd
-// element count leaves one scalar tail element for thread 0 of CTA 0.
-template <class F2, class F1>
-__device__ __forceinline__ void elemwise(int64_t n, F2 body2, F1 body1) {
-  const int64_t n2 = n >> 1;
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n2; x += (int64_t)gridDim.x * kT) body2(x);
-  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) body1(n - 1);
-}
+// = 16 CTAs per SM; every thread loads kU pairs (one grid stride apart) before it
+// computes and stores any of them, so enough loads are in flight to stream at the
+// HBM rate (one pair per iteration left the fused epilogue at 1.6 TB/s: ncu
+// long-scoreboard 197 cycles per issue).  An odd element count leaves one scalar
+// tail element for thread 0 of CTA 0.
+constexpr int kU = 4;
 __device__ __forceinline__ double2 ld2(const double* p, int64_t x) { return reinterpret_cast<const double2*>(p)[x]; }
 __device__ __forceinline__ void st2(double* p, int64_t x, double a, double b) {
   reinterpret_cast<double2*>(p)[x] = make_double2(a, b);
 }
 __device__ __forceinline__ double prox0(double v) { return v > 0.0 ? v : 0.0; }
+#define ABL_LOOP_BEGIN                                                               \
+  const int64_t n2 = n >> 1, stride = (int64_t)gridDim.x * kT;                       \
+  for (int64_t x0 = blockIdx.x * (int64_t)kT + threadIdx.x; x0 < n2; x0 += kU * stride) {
+#define ABL_LOOP_END }
+#define ABL_FOR_K _Pragma("unroll") for (int k = 0; k < kU; k++)
+#define ABL_X const int64_t x = x0 + k * stride; if (x < n2)
+#define ABL_TAIL if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0)
 
 // ---- unfused element-wise steps of Alg. 2 (one call per operation)
 __global__ void k_prox(const double* __restrict__ Ht, const double* __restrict__ U, double* __restrict__ H, int64_t n) {
-  elemwise(n, [&](int64_t x) {                        // Alg. 2 l.7 with the indicator of R_+
-    const double2 h = ld2(Ht, x), u = ld2(U, x);
-    st2(H, x, prox0(h.x - u.x), prox0(h.y - u.y));
-  }, [&](int64_t x) { H[x] = prox0(Ht[x] - U[x]); });
+  ABL_LOOP_BEGIN                                     // Alg. 2 l.7 with the indicator of R_+
+    double2 h[kU], u[kU];
+    ABL_FOR_K { ABL_X { h[k] = ld2(Ht, x); u[k] = ld2(U, x); } }
+    ABL_FOR_K { ABL_X st2(H, x, prox0(h[k].x - u[k].x), prox0(h[k].y - u[k].y)); }
+  ABL_LOOP_END
+  ABL_TAIL H[n - 1] = prox0(Ht[n - 1] - U[n - 1]);
 }
 __global__ void k_dual(const double* __restrict__ H, const double* __restrict__ Ht, double* __restrict__ U, int64_t n) {
-  elemwise(n, [&](int64_t x) {                        // Alg. 2 l.8
-    const double2 h = ld2(H, x), t = ld2(Ht, x), u = ld2(U, x);
-    st2(U, x, u.x + h.x - t.x, u.y + h.y - t.y);
-  }, [&](int64_t x) { U[x] = U[x] + H[x] - Ht[x]; });
+  ABL_LOOP_BEGIN                                     // Alg. 2 l.8
+    double2 h[kU], t[kU], u[kU];
+    ABL_FOR_K { ABL_X { h[k] = ld2(H, x); t[k] = ld2(Ht, x); u[k] = ld2(U, x); } }
+    ABL_FOR_K { ABL_X st2(U, x, u[k].x + h[k].x - t[k].x, u[k].y + h[k].y - t[k].y); }
+  ABL_LOOP_END
+  ABL_TAIL U[n - 1] = U[n - 1] + H[n - 1] - Ht[n - 1];
 }
 
 __device__ __forceinline__ void block_store4(double a, double b, double c, double d, double* __restrict__ part) {
@@ -146,17 +155,20 @@ __device__ __forceinline__ void acc4(double h, double ht, double h0, double u, d
   r += e1 * e1; s += e2 * e2; nh += h * h; nu += u * u;
 }
 // residual sums of the baseline (the norms of Alg. 2 l.9, one pass over the four matrices)
-// (explicit loops: accumulators captured by reference in a lambda went to local memory)
 __global__ void k_resid(const double* __restrict__ H, const double* __restrict__ Ht, const double* __restrict__ H0,
                         const double* __restrict__ U, int64_t n, double* __restrict__ part) {
   double r = 0, s = 0, h = 0, u = 0;
-  const int64_t n2 = n >> 1;
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n2; x += (int64_t)gridDim.x * kT) {
-    const double2 a = ld2(H, x), t = ld2(Ht, x), z = ld2(H0, x), v = ld2(U, x);
-    acc4(a.x, t.x, z.x, v.x, r, s, h, u);
-    acc4(a.y, t.y, z.y, v.y, r, s, h, u);
-  }
-  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) acc4(H[n - 1], Ht[n - 1], H0[n - 1], U[n - 1], r, s, h, u);
+  ABL_LOOP_BEGIN
+    double2 a[kU], t[kU], z[kU], v[kU];
+    ABL_FOR_K { ABL_X { a[k] = ld2(H, x); t[k] = ld2(Ht, x); z[k] = ld2(H0, x); v[k] = ld2(U, x); } }
+    ABL_FOR_K {
+      ABL_X {
+        acc4(a[k].x, t[k].x, z[k].x, v[k].x, r, s, h, u);
+        acc4(a[k].y, t[k].y, z[k].y, v[k].y, r, s, h, u);
+      }
+    }
+  ABL_LOOP_END
+  ABL_TAIL acc4(H[n - 1], Ht[n - 1], H0[n - 1], U[n - 1], r, s, h, u);
   block_store4(r, s, h, u, part);
 }
 
@@ -165,10 +177,12 @@ __global__ void k_resid(const double* __restrict__ H, const double* __restrict__
 __global__ void k_fused_T(const double* __restrict__ M, const double* __restrict__ H, const double* __restrict__ U,
                           const double* __restrict__ consts, double* __restrict__ T, int64_t n) {
   const double rho = consts[1];
-  elemwise(n, [&](int64_t x) {
-    const double2 m = ld2(M, x), h = ld2(H, x), u = ld2(U, x);
-    st2(T, x, m.x + rho * (h.x + u.x), m.y + rho * (h.y + u.y));
-  }, [&](int64_t x) { T[x] = M[x] + rho * (H[x] + U[x]); });
+  ABL_LOOP_BEGIN
+    double2 m[kU], h[kU], u[kU];
+    ABL_FOR_K { ABL_X { m[k] = ld2(M, x); h[k] = ld2(H, x); u[k] = ld2(U, x); } }
+    ABL_FOR_K { ABL_X st2(T, x, m[k].x + rho * (h[k].x + u[k].x), m[k].y + rho * (h[k].y + u[k].y)); }
+  ABL_LOOP_END
+  ABL_TAIL T[n - 1] = M[n - 1] + rho * (H[n - 1] + U[n - 1]);
 }
 // prox + dual + residual partials in one pass; H0 is the incoming H (no copy)
 __device__ __forceinline__ void epi1(double ht, double h0, double u0, double& hn, double& un, double& r, double& s,
@@ -180,16 +194,20 @@ __device__ __forceinline__ void epi1(double ht, double h0, double u0, double& hn
 __global__ void k_fused_epi(const double* __restrict__ Ht, double* __restrict__ H, double* __restrict__ U, int64_t n,
                             double* __restrict__ part) {
   double r = 0, s = 0, h = 0, u = 0;
-  const int64_t n2 = n >> 1;
-  for (int64_t x = blockIdx.x * (int64_t)kT + threadIdx.x; x < n2; x += (int64_t)gridDim.x * kT) {
-    const double2 t = ld2(Ht, x), h0 = ld2(H, x), u0 = ld2(U, x);
-    double a, b, c, d;
-    epi1(t.x, h0.x, u0.x, a, c, r, s, h, u);
-    epi1(t.y, h0.y, u0.y, b, d, r, s, h, u);
-    st2(H, x, a, b);
-    st2(U, x, c, d);
-  }
-  if ((n & 1) && blockIdx.x == 0 && threadIdx.x == 0) {
+  ABL_LOOP_BEGIN
+    double2 t[kU], h0[kU], u0[kU];
+    ABL_FOR_K { ABL_X { t[k] = ld2(Ht, x); h0[k] = ld2(H, x); u0[k] = ld2(U, x); } }
+    ABL_FOR_K {
+      ABL_X {
+        double a, b, c, d;
+        epi1(t[k].x, h0[k].x, u0[k].x, a, c, r, s, h, u);
+        epi1(t[k].y, h0[k].y, u0[k].y, b, d, r, s, h, u);
+        st2(H, x, a, b);
+        st2(U, x, c, d);
+      }
+    }
+  ABL_LOOP_END
+  ABL_TAIL {
     double a, c;
     epi1(Ht[n - 1], H[n - 1], U[n - 1], a, c, r, s, h, u);
     H[n - 1] = a;

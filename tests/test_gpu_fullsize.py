@@ -121,3 +121,18 @@ def test_fullsize_delicious_mttkrp_sampled_rows(delicious):
         assert normwise(got, want) <= TOL, n
         assert not torch.isnan(M).any().item()
         del M
+
+
+def test_fullsize_delicious_one_outer_iteration(delicious):
+    """configs[3] at full size in the bench's launch configuration (default layout:
+    hot-row tables, L2-blocked mode 4; eps = 0, 10 passes): one outer iteration end to
+    end against the oracle (~40 s of CPU work) -- fit, factors and lambda <= 1e-6."""
+    B, c, X, ref, F = delicious
+    Fd = [torch.from_numpy(f.copy()).cuda() for f in F]
+    lam = torch.zeros(c.R, dtype=torch.float64, device="cuda")
+    rep = B.cstf_factorize(X, Fd, lam, B.make_opts(c.R, outer_iters=1, tol=0.0, max_iter=10))
+    orc = oracle.factorize(ref, F, outer_iters=1, tol=0.0, max_iter=10)
+    assert abs(rep["fit"][0] - orc["fit"][0]) <= 1e-6 * abs(orc["fit"][0])
+    for a, b in zip(Fd, orc["factors"]):
+        assert normwise(a.cpu().numpy(), b) <= 1e-6
+    assert normwise(lam.cpu().numpy(), orc["lam"][-1]) <= 1e-6

@@ -28,6 +28,20 @@ namespace {
 
 constexpr int kWarps = 8;  // per CTA
 
+// Resident CTAs per SM of the fast kernel (its register budget) by average nonzeros
+// per row: < 16 -> 4 (64 registers: row flushes dominate, latency hiding needs
+// warps), < 64 -> 3 for R = 32 / 64 (80 registers; Delicious mode 3, 56 per row:
+// 10.81 -> 9.91 ms), else 2 (long rows).  CSTF_MTTKRP_MINB=2/3/4 forces (experiments).
+int mttkrp_minb(int64_t nnz, int64_t rows, int R) {
+  if (const char* e = getenv("CSTF_MTTKRP_MINB")) {
+    const int v = atoi(e);
+    if (v == 2 || v == 4 || (v == 3 && (R == 32 || R == 64))) return v;
+  }
+  if (nnz < 16 * rows) return 4;
+  if (nnz < 64 * rows) return (R == 32 || R == 64) ? 3 : 4;
+  return 2;
+}
+
 struct MArgs {
   const int64_t* rowptr;
   const char* rec;
@@ -408,9 +422,12 @@ bool launch_tiled_r(const MArgs& a, int grid, cudaStream_t st) {
 
 template <int NOTHER, int RECB>
 bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, bool hot) {
-  // short rows (few nonzeros per row): row flushes dominate and latency hiding
-  // needs more warps -> the 4-CTA/SM register budget; long rows -> 2 CTAs/SM
-  const bool short_rows = a.nnz < 64 * (a.I - a.rbase);
+  // CTAs per SM by nonzeros per row (mttkrp_minb): short rows -- row flushes dominate,
+  // latency hiding needs warps -- 4 (64 registers); medium rows (R = 32 / 64) 3 (80);
+  // long rows 2 (128)
+  const int minb = mttkrp_minb(a.nnz, a.I - a.rbase, a.R);
+  const bool short_rows = minb == 4;
+  const bool mid_rows = minb == 3;
   if (tiled) {
     switch (a.R) {     // slab = 256 rows x R doubles: 2 KB .. 128 KB
       case 8: return launch_tiled_r<NOTHER, RECB, 8>(a, grid, st);
@@ -423,6 +440,7 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
 #define GCASE(RR, GG)                                                                   \
   if (a.R == RR && gl == GG) {                                                      \
     if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4, GG><<<grid, kWarps * 32, 0, st>>>(a); \
+    else if (mid_rows) k_mttkrp_fast<NOTHER, RR, RECB, 3, GG><<<grid, kWarps * 32, 0, st>>>(a); \
     else k_mttkrp_fast<NOTHER, RR, RECB, 2, GG><<<grid, kWarps * 32, 0, st>>>(a);          \
     return true;                                                                        \
   }
@@ -433,6 +451,7 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
 #define HCASE(RR)                                                                              \
   case RR:                                                                                     \
     if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4, 0, true><<<grid, kWarps * 32, 0, st>>>(a); \
+    else if (mid_rows) k_mttkrp_fast<NOTHER, RR, RECB, 3, 0, true><<<grid, kWarps * 32, 0, st>>>(a); \
     else k_mttkrp_fast<NOTHER, RR, RECB, 2, 0, true><<<grid, kWarps * 32, 0, st>>>(a);           \
     return true;
       HCASE(16) HCASE(32) HCASE(64)
@@ -446,8 +465,15 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
     if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4><<<grid, kWarps * 32, 0, st>>>(a); \
     else k_mttkrp_fast<NOTHER, RR, RECB, 2><<<grid, kWarps * 32, 0, st>>>(a);           \
     return true;
-    CASE(2) CASE(4) CASE(8) CASE(16) CASE(32) CASE(64) CASE(128)
+#define CASE3(RR)                                                                    \
+  case RR:                                                                           \
+    if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4><<<grid, kWarps * 32, 0, st>>>(a); \
+    else if (mid_rows) k_mttkrp_fast<NOTHER, RR, RECB, 3><<<grid, kWarps * 32, 0, st>>>(a); \
+    else k_mttkrp_fast<NOTHER, RR, RECB, 2><<<grid, kWarps * 32, 0, st>>>(a);           \
+    return true;
+    CASE(2) CASE(4) CASE(8) CASE(16) CASE3(32) CASE3(64) CASE(128)
 #undef CASE
+#undef CASE3
     default: return false;
   }
 }
@@ -570,8 +596,7 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     if (B == 1) return fail(CSTF_ERR_OUT_OF_MEMORY, "MTTKRP partial rows of one L2 block (set CSTF_L2_BLOCK=0)");
     B = (B + 1) / 2;
   }
-  const bool short_rows = nnz < 64 * ms.Ivirt;        // = launch_fast's CTA budget
-  const int ctas = di.sms * (short_rows ? 4 : 2);      // resident CTAs only
+  const int ctas = di.sms * mttkrp_minb(nnz, ms.Ivirt, R);   // resident CTAs only (= launch_fast's budget)
   // chunk: the window in flight (resident warps x chunk) about half a block
   int64_t chunk = (nnz / std::max<int64_t>(nblk, 1)) / (2 * (int64_t)ctas * kWarps);
   chunk = std::min<int64_t>(1024, std::max<int64_t>(256, (chunk + 31) / 32 * 32));
@@ -904,7 +929,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
       CSTF_TRY(w.queue.ensure(8));
       CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
       a.queue = w.queue.as<unsigned long long>();
-      grid = std::min(grid, di.sms * (nnz < 64 * ms.Ivirt ? 4 : 2));
+      grid = std::min(grid, di.sms * mttkrp_minb(nnz, ms.Ivirt, R));
     }
   }
   {

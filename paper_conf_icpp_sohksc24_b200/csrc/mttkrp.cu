@@ -31,14 +31,16 @@ constexpr int kWarps = 8;  // per CTA
 // Resident CTAs per SM of the fast kernel (its register budget) by average nonzeros
 // per row: < 16 -> 4 (64 registers: row flushes dominate, latency hiding needs
 // warps), < 64 -> 3 for R = 32 / 64 (80 registers; Delicious mode 3, 56 per row:
-// 10.81 -> 9.91 ms), else 2 (long rows).  CSTF_MTTKRP_MINB=2/3/4 forces (experiments).
-int mttkrp_minb(int64_t nnz, int64_t rows, int R) {
+// 10.81 -> 10.0 ms), else 2 (long rows).  Virtual rows of L2-blocked copies (`tiled`)
+// keep 4 below 64 (Amazon, ~20 per virtual row: 531 -> 592 ms with 3).
+// CSTF_MTTKRP_MINB=2/3/4 forces (experiments).
+int mttkrp_minb(int64_t nnz, int64_t rows, int R, bool tiled) {
   if (const char* e = getenv("CSTF_MTTKRP_MINB")) {
     const int v = atoi(e);
     if (v == 2 || v == 4 || (v == 3 && (R == 32 || R == 64))) return v;
   }
   if (nnz < 16 * rows) return 4;
-  if (nnz < 64 * rows) return (R == 32 || R == 64) ? 3 : 4;
+  if (nnz < 64 * rows) return (!tiled && (R == 32 || R == 64)) ? 3 : 4;
   return 2;
 }
 
@@ -60,6 +62,7 @@ struct MArgs {
   double* carry;        // [nchunks][R]
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
+  int l2blocked;        // launch over an L2-blocked copy (rows are virtual rows)
 };
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
@@ -425,7 +428,7 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
   // CTAs per SM by nonzeros per row (mttkrp_minb): short rows -- row flushes dominate,
   // latency hiding needs warps -- 4 (64 registers); medium rows (R = 32 / 64) 3 (80);
   // long rows 2 (128)
-  const int minb = mttkrp_minb(a.nnz, a.I - a.rbase, a.R);
+  const int minb = mttkrp_minb(a.nnz, a.I - a.rbase, a.R, a.l2blocked != 0);
   const bool short_rows = minb == 4;
   const bool mid_rows = minb == 3;
   if (tiled) {
@@ -596,7 +599,8 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     if (B == 1) return fail(CSTF_ERR_OUT_OF_MEMORY, "MTTKRP partial rows of one L2 block (set CSTF_L2_BLOCK=0)");
     B = (B + 1) / 2;
   }
-  const int ctas = di.sms * mttkrp_minb(nnz, ms.Ivirt, R);   // resident CTAs only (= launch_fast's budget)
+  const int ctas = di.sms * mttkrp_minb(nnz, ms.Ivirt, R, true);   // resident CTAs only (= launch_fast's budget)
+  a.l2blocked = 1;
   // chunk: the window in flight (resident warps x chunk) about half a block
   int64_t chunk = (nnz / std::max<int64_t>(nblk, 1)) / (2 * (int64_t)ctas * kWarps);
   chunk = std::min<int64_t>(1024, std::max<int64_t>(256, (chunk + 31) / 32 * 32));
@@ -794,6 +798,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.wstart = nullptr;
   a.ckb = nullptr;
   a.queue = nullptr;
+  a.l2blocked = 0;
   a.pbase = 0;
   a.cbase = 0;
   a.rbase = 0;
@@ -929,7 +934,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
       CSTF_TRY(w.queue.ensure(8));
       CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
       a.queue = w.queue.as<unsigned long long>();
-      grid = std::min(grid, di.sms * mttkrp_minb(nnz, ms.Ivirt, R));
+      grid = std::min(grid, di.sms * mttkrp_minb(nnz, ms.Ivirt, R, false));
     }
   }
   {

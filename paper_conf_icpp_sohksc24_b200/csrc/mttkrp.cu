@@ -30,7 +30,7 @@ constexpr int kWarps = 8;  // per CTA
 
 // Resident CTAs per SM of the fast kernel (its register budget) by average nonzeros
 // per row: < 16 -> 4 (64 registers: row flushes dominate, latency hiding needs
-// warps), < 64 -> 3 for R = 32 / 64 (80 registers; Delicious mode 3, 56 per row:
+// warps), < 64 -> 3 for R = 32 / 64 (80 registers; Delicious mode 2, 56 per row:
 // 10.81 -> 10.0 ms), else 2 (long rows).  Virtual rows of L2-blocked copies (`tiled`)
 // keep 4 below 64 (Amazon, ~20 per virtual row: 531 -> 592 ms with 3).
 // CSTF_MTTKRP_MINB=2/3/4 forces (experiments).

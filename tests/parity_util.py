@@ -35,3 +35,27 @@ def compare_iteration_counts(gpu_iters, orc, eps):
                 return n, (t, m, mu)
             n += 1
     return n, None
+
+
+def compare_all_iteration_counts(gpu_iters, orc, eps):
+    """Every (outer iteration, mode) pair: the counts are equal, or the mismatch is a
+    tie (U2: |mu| < TIE_MARGIN at the oracle's pass min(k_gpu, k_orc)).  Unlike
+    compare_iteration_counts this keeps comparing after a tie (both trajectories
+    stay within rounding of each other once they sit at the fixed point).
+    Returns (n_equal, n_ties)."""
+    oi = orc["iters"]
+    tr = orc["trace"]
+    assert gpu_iters.shape == oi.shape, (gpu_iters.shape, oi.shape)
+    eq = ties = 0
+    for t in range(oi.shape[0]):
+        for m in range(oi.shape[1]):
+            kg, ko = int(gpu_iters[t, m]), int(oi[t, m])
+            if kg == ko:
+                eq += 1
+                continue
+            mu = stop_margin(tr[t, m, min(kg, ko) - 1], eps)
+            assert abs(mu) < TIE_MARGIN, (
+                f"ADMM iteration count differs at outer {t} mode {m}: gpu {kg} oracle {ko}, "
+                f"margin {mu:.3e} is not a tie")
+            ties += 1
+    return eq, ties

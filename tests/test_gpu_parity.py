@@ -10,7 +10,7 @@ import pytest
 
 import datagen
 import oracle
-from parity_util import compare_iteration_counts
+from parity_util import compare_all_iteration_counts, compare_iteration_counts
 
 torch = pytest.importorskip("torch")
 pytestmark = pytest.mark.gpu
@@ -333,18 +333,23 @@ def run_both(B, dims, idx, vals, R, start, outer=10, tol=1e-2, max_iter=10, warm
 
 
 def test_factorize_planted_tiny(B):
-    """configs[0]: fit after 10 outer iterations within 1e-6 and equal ADMM counts."""
+    """configs[0]: fit after 10 outer iterations within 1e-6; every one of the 30 ADMM
+    iteration counts equals the oracle's or differs at a tie (U2: |mu| < 1e-12 at the
+    decisive pass -- the planted tensor is fitted exactly from outer iteration 6 on and
+    its stop test then compares rounding noise, r, s, nU ~ 1e-31); factors <= 1e-6."""
     p = datagen.planted_tiny(1)
     start = datagen.perturbed_start(p, 1)
     orc, gpu, F, lam = run_both(B, p.dims, p.idx, p.vals, p.R, start)
     assert gpu["outer_done"] == 10
     n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
     assert n >= 15            # the first five outer iterations are decided well away from ties
+    eq, ties = compare_all_iteration_counts(gpu["iters"], orc, 1e-2)
+    assert eq + ties == 30 and eq >= 20, (eq, ties)
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
     assert gpu["fit"][-1] >= 1 - 1e-6          # recovery (the 1e-8 gate is the oracle's pin P8)
-    if tie is None:
-        for a, b in zip(F, orc["factors"]):
-            assert normwise(a, b) <= 1e-6
+    for a, b in zip(F, orc["factors"]):
+        assert normwise(a, b) <= 1e-6
+    assert normwise(lam, orc["lam"][-1]) <= 1e-6
 
 
 @pytest.mark.parametrize("cfg,scale,R", [("nell2", 40, 16), ("enron", 40, 8), ("delicious", 2000, 8)])

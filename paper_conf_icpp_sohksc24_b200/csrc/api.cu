@@ -341,7 +341,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
     }
   } hotg;
   hotg.st = st;
-  if (!dist) CSTF_TRY(hot_persist_begin(X, hotg.p));
+  CSTF_TRY(hot_persist_begin(X, hotg.p));
   double* G = w.grams.as<double>();
   double* lam = w.lam.as<double>();
   double* lam_scratch = lam + (size_t)N * R;
@@ -463,7 +463,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       }
       if (rep && rep->admm_iters) rep->admm_iters[t * N + n] = iters;
       tm.end(n, CSTF_PHASE_UPDATE);
-      // the hot-row table of factor n follows its update (the next MTTKRPs read it)
+      // the hot-row table of factor n follows its update (the next MTTKRPs read it);
+      // distributed: from the full replica, once every rank's rows are in (below)
       if (!dist) CSTF_TRY(hot_refresh(X, n, Hn, R, st));
       // a7 (when not fused): raw Gram; a6: lambda and the normalised Gram
       if (!fused) {
@@ -483,6 +484,7 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
       CSTF_TRY(comm_allreduce_f64(comm, Gn, (size_t)R * R, st));
       CSTF_TRY(gram_to_lambda(Gn, R, lam + n * R, st));
       tm.end(n, CSTF_PHASE_NORMALIZE);
+      if (dist) CSTF_TRY(hot_refresh(X, n, fac[n], R, st));
       if (hout && t == o->outer_iters - 1) {   // final factor n: normalised copy to the host now
         double* sn = w.stage.as<double>() + stage_off[n];
         CSTF_CUDA(cudaMemcpyAsync(sn, fac[n], (size_t)Ifull[n] * R * 8, cudaMemcpyDeviceToDevice, st));

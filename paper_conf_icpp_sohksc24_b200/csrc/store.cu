@@ -398,6 +398,9 @@ void decide_l2_block(ModeStore& ms, int N, int64_t nloc, int64_t Iloc, const int
 // ranks (cstf_partition_rows); all indices are relabelled to
 // owner * B_n + local, and this rank keeps, for every mode n, the nonzeros whose
 // mode-n row it owns, with the row index local to its block.
+cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap, double* cov, cudaStream_t st,
+                       const int64_t* dims_override = nullptr);
+
 cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int64_t nout, DevBuf& tmp,
                               cudaStream_t st) {
   const int N = X->N, P = X->nranks, rk = X->rank;
@@ -429,6 +432,16 @@ cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int
       CSTF_LAUNCHED();
     }
     CSTF_CUDA(cudaStreamSynchronize(st));
+  }
+  // hot-row tables over the internal labels of the replicated factors (same rule as the
+  // single-GPU store; every rank selects the same rows: the counts are global)
+  DevBuf hmap[8];
+  {
+    double cov[8];
+    int64_t Iint[8];
+    for (int k = 0; k < N; k++) Iint[k] = (int64_t)P * X->rows_per_rank[k];
+    static const bool kblock_env = getenv("CSTF_KBLOCK") && atoi(getenv("CSTF_KBLOCK")) > 0;
+    if (!kblock_env) CSTF_TRY(decide_hot(X, lab_idx, nout, hmap, cov, st, Iint));
   }
   const int recb = record_bytes(N);
   for (int n = 0; n < N; n++) {
@@ -522,6 +535,15 @@ cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int
     ra.nslots = N - 1;
     ra.recb = recb;
     for (int q = 0; q < N - 1; q++) ra.idx[q] = kk[q + 1].as<int32_t>();
+    ms.hotmask = 0;
+    {
+      const bool slab_window = ms.tiled && ns / std::max<int64_t>(ms.nblk, 1) >= ((int64_t)16 << 20);
+      for (int q = 0; q < N - 1 && !slab_window; q++)
+        if (X->hot_cnt[ms.other[q]] > 0 && !(ms.tiled && q == ms.tslot)) {
+          ra.hmap[q] = hmap[ms.other[q]].as<int32_t>();
+          ms.hotmask |= 1 << q;
+        }
+    }
     if (ns) {
       k_make_records<<<grid_for(ns), kThreads, 0, st>>>(ra, vv.as<double>(), pm.as<uint32_t>(), ns, ms.rec.as<char>());
       CSTF_LAUNCHED();
@@ -541,7 +563,10 @@ cstf_status build_partitioned(cstf_tensor* X, DevBuf* c_idx, DevBuf& c_vals, int
 // row to its hot slot or -1 and is used while the mode copies are built.
 // Also fills cov[k] (all factors larger than half the L2 at R = 32): the share of the
 // nonzeros on the factor's L2-capacity hottest rows, for the skew-aware L2-block choice.
-cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap, double* cov, cudaStream_t st) {
+// dims_override (partitioned store): the internal (padded) factor lengths, c_idx the
+// internal labels.
+cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap, double* cov, cudaStream_t st,
+                       const int64_t* dims_override) {
   const int N = X->N;
   X->hot_total = 0;
   for (int k = 0; k < N; k++) cov[k] = 1.0;
@@ -557,7 +582,7 @@ cstf_status decide_hot(cstf_tensor* X, DevBuf* c_idx, int64_t nout, DevBuf* hmap
   for (int k = 0; k < N; k++) {
     X->hot_off[k] = (int64_t)all.size();
     X->hot_cnt[k] = 0;
-    const int64_t I = X->dims[k];
+    const int64_t I = dims_override ? dims_override[k] : X->dims[k];
     const bool big = forced > 0 ? I > 2 * forced : I * 256 > (int64_t)device_info().l2 / 2;
     if (!big || nout == 0) continue;
     DevBuf cnt;

@@ -78,15 +78,19 @@ def run(tmp_path, nproc, case, port, comm="host"):
     (1, ("enron", 60, 8, 1e-2, 5), 29617, "nccl"),
     (2, ("nell2", 40, 32, 0.0, 4), 29618, "blk"),          # L2-blocked partitioned copies (forced)
     (3, ("enron", 60, 16, 1e-2, 5), 29619, "blk"),
+    (2, ("delicious", 1000, 32, 0.0, 3), 29620, "hot"),   # hot-row tables over internal labels (forced)
+    (3, ("delicious", 1000, 16, 1e-2, 4), 29622, "hot"),
 ])
 def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port, peer, monkeypatch):
     """peer: CSTF_PEER_STORE for the host communicator, or "nccl" (one rank: the
     NCCL transport -- dlopen, unique id, init, all-reduce, all-gather -- and the
     partitioned layout with P = 1, the only NCCL job one GPU can run)."""
     comm = "nccl" if peer == "nccl" else "host"
-    monkeypatch.setenv("CSTF_PEER_STORE", "1" if peer in ("nccl", "blk") else peer)
+    monkeypatch.setenv("CSTF_PEER_STORE", "1" if peer in ("nccl", "blk", "hot") else peer)
     if peer == "blk":
         monkeypatch.setenv("CSTF_L2_BLOCK_ROWS", "64")
+    if peer == "hot":
+        monkeypatch.setenv("CSTF_HOT_ROWS", "150")
     res = run(tmp_path, nproc, case, port, comm)
     r0 = res[0]
     for rk in range(1, nproc):          # every rank took the same decisions
@@ -94,7 +98,7 @@ def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port, peer,
     assert r0["fit_rel"] <= 1e-6
     if peer == "blk":
         assert all(max(res[rk]["nblk"]) > 1 for rk in range(nproc))     # some mode copy L2-blocked
-    if nproc > 1 and peer in ("1", "blk") and case[3] == 0.0 and case[2] <= 32:
+    if nproc > 1 and peer in ("1", "blk", "hot") and case[3] == 0.0 and case[2] <= 32:
         assert r0["comm_ms"] == 0.0          # no separate all-gather ran: rows were peer-stored
     if not r0["tie"]:
         assert r0["fac_rel"] <= 1e-6 and r0["lam_rel"] <= 1e-6

@@ -213,6 +213,41 @@ def admm_ablation(B, cfg, R, stream, reps=3):
     return out
 
 
+def admm_streaming_probe(B, cfg, R, stream, hbm_peak, reps=3):
+    """The metric's literal "ADMM update HBM GB/s": libcstf's one-launch-per-pass
+    ADMM kernel (v1: reads M, H, U and writes H, U every pass = 40 I R bytes per
+    pass) on the largest mode of this workload, 10 passes, CUDA events.  The bench's
+    own update is the row-resident kernel (FP64-bound; it moves those bytes once)."""
+    import torch
+    n = int(np.argmax(cfg.dims))
+    I = cfg.dims[n]
+    f = datagen.uniform(cfg.seed, 60, 256 * R).reshape(256, R)
+    f = f / np.linalg.norm(f, axis=0)
+    g = torch.zeros(R, R, dtype=torch.float64, device="cuda")
+    B.cstf_gram(torch.from_numpy(f).cuda(), g)
+    S = g * g                                                   # Hadamard of two unit-diagonal Grams
+    M = torch.rand(I, R, dtype=torch.float64, device="cuda")
+    H = torch.rand(I, R, dtype=torch.float64, device="cuda")
+    U = torch.zeros_like(H)
+    B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=B.CSTF_ADMM_STREAMING)
+    ts = []
+    for _ in range(reps):
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        a.record(stream)
+        B.cstf_admm_update(M, S, H, U, tol=0.0, max_iter=10, variant=B.CSTF_ADMM_STREAMING)
+        b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b))
+    ms = float(np.median(ts))
+    byts = 10 * cm.admm_bytes(I, R)
+    del M, H, U
+    torch.cuda.empty_cache()
+    return {"mode": n, "rows": I, "passes": 10, "ms": ms, "gbs": byts / (ms * 1e-3) / 1e9,
+            "frac_of_hbm": byts / (ms * 1e-3) / 1e9 / hbm_peak,
+            "note": "k_admm_dmma with one launch per pass (CSTF_ADMM_STREAMING), 40 I R bytes per pass"}
+
+
 def relaunch_under_torchrun(n):
     """--gpus N > 1 without a torchrun environment: run this command again as N ranks
     (one process per GPU, rendezvous on 127.0.0.1)."""
@@ -240,6 +275,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-streaming-probe", action="store_true",
+                    help="skip timing the one-launch-per-pass ADMM kernel on the largest mode")
     ap.add_argument("--comm", choices=["nccl", "host"], default="nccl",
                     help="N > 1 transport: nccl (one GPU per rank, the product path) or host (gloo "
                          "host callbacks; ranks may share one GPU -- validates the multi-rank path, "
@@ -423,6 +460,8 @@ def main():
         line["e2e"] = {"value": e2e_s, "unit": "s", "h2d_bytes_per_step": fac_bytes,
                        "d2h_bytes_per_step": fac_bytes + R * 8 + 8,
                        "note": "cstf_factorize_host: initial factors H2D, 1 outer iteration, factors+lambda+fit D2H"}
+    if world == 1 and not args.no_streaming_probe:
+        line["admm_update_gbs"]["streaming_v1"] = admm_streaming_probe(B, cfg, R, stream, peaks["hbm_gbs"])
     if args.ablation and world == 1:
         line["ablation"] = admm_ablation(B, cfg, R, stream)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

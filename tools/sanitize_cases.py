@@ -24,7 +24,7 @@ def cu(a):
 
 def main():
     torch.cuda.set_device(0)
-    which = sys.argv[1:] or ["planted", "fixed", "l2block", "hot", "admm64", "hals_mu", "ablation"]
+    which = sys.argv[1:] or ["planted", "fixed", "l2block", "hot", "admm64", "hals_mu", "partitioned", "ablation"]
     if "planted" in which:
         p = datagen.planted_tiny(1)
         X = B.cstf_tensor_load_coo(p.dims, p.idx, p.vals)
@@ -81,6 +81,16 @@ def main():
         B.cstf_hals_update(cu(M), cu(S), cu(H), sweeps=2)
         B.cstf_mu_update(cu(M), cu(S), cu(H), sweeps=2)
         print("hals_mu ok", flush=True)
+    if "partitioned" in which:        # one-part loopback communicator: partitioned store, hot rows, agreement
+        os.environ["CSTF_HOT_ROWS"] = "100"
+        comm = B.cstf_comm_loopback(1)[0]
+        dims = (60, 2000, 700, 20)
+        idx, vals = datagen.coo(dims, (2, 2, 3, 1), 30000, 52)
+        X = B.cstf_tensor_load_coo(dims, idx, vals, comm=comm)
+        F = [cu(f) for f in datagen.init_factors(dims, 32, 9)]
+        B.cstf_factorize(X, F, cu(np.zeros(32)), B.make_opts(32, outer_iters=2, tol=0.0, max_iter=4), comm=comm)
+        del os.environ["CSTF_HOT_ROWS"]
+        print("partitioned ok", flush=True)
     if "ablation" in which:
         from paper_conf_icpp_sohksc24_b200 import ablation as AB
         rng = np.random.default_rng(3)

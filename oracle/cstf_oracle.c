@@ -19,9 +19,11 @@
  *   O9/O11 oracle_factorize Alg. 1 (L476-506) with readings D4, D6, D11, D13
  * Readings D1-D20 are listed in DESIGN.md.
  *
- * Parity status: see DESIGN.md "Oracle pins".  Summation order inside MTTKRP,
- * Gram and the residual sums differs from the GPU's; that difference is
- * "parity unpinned" (U1) and is bounded by the tolerances in tests/.
+ * Parity status: every function above is pinned (DESIGN.md "Oracle pins",
+ * tests/test_oracle_pins.py); none is "parity unpinned".  The summation order
+ * inside MTTKRP, Gram and the residual sums differs from the GPU's (U1): a
+ * rounding-order difference between two pinned implementations, bounded by
+ * the tolerances in tests/, not a function without a pin.
  *
  * Determinism: every reduction uses fixed 4096-row blocks summed in block
  * order, so results are bitwise identical for any OMP_NUM_THREADS (pin P11).

@@ -1,6 +1,7 @@
-"""Full-size parity at the bench configuration (configs[1], NELL-2-shaped,
+"""Full-size parity at configs[1] (NELL-2-shaped,
 77M nonzeros, R = 32, eps = 0, 10 inner passes) on sampled outputs the oracle
-can compute one by one, plus one complete outer iteration end to end."""
+can compute one by one, plus one complete outer iteration end to end; the same
+at configs[3] (Delicious-shaped, 140M nonzeros: the bench default) below."""
 import numpy as np
 import pytest
 

@@ -1,0 +1,89 @@
+"""Full-size parity at configs[4] (Amazon-reviews-shaped, 4.8M x 1.8M x 1.8M,
+1.7B nonzeros, R = 64; Table 2, ranks L907-908) on sampled
+outputs the oracle computes one by one.  Only the full size exercises the
+default L2-blocked layout with one launch per block under a persisting L2
+window (blocks of >= 16M nonzeros) and the R = 64 row-resident ADMM with its
+row-group prefetch over millions of rows.
+
+The oracle never sees the whole tensor: for each sampled output row it gets the
+sub-tensor of the nonzeros whose mode-n index is that row (MTTKRP rows are
+independent, Fig. 2), coalesced by the oracle itself.
+
+Opt-in (several minutes, ~40 GB of host memory): CSTF_TEST_AMAZON=1."""
+import os
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(os.environ.get("CSTF_TEST_AMAZON") != "1",
+                                 reason="full-size Amazon parity is opt-in (CSTF_TEST_AMAZON=1)")]
+
+TOL = 1e-9
+
+
+def normwise(a, b):
+    den = np.max(np.abs(b))
+    return float(np.max(np.abs(np.asarray(a) - np.asarray(b))) / (den if den > 0 else 1.0))
+
+
+@pytest.fixture(scope="module")
+def amazon():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_icpp_sohksc24_b200 import binding as B
+    c = datagen.CONFIGS["amazon"]
+    idx, vals = c.generate()
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    F = datagen.init_factors(c.dims, c.R, c.seed)
+    yield B, c, X, idx, vals, F
+    X.free()
+
+
+def sub_tensor(c, idx, vals, n, rows):
+    """The oracle's coalesced tensor of the nonzeros whose mode-n index is in rows."""
+    sel = np.zeros(c.dims[n], dtype=bool)
+    sel[rows] = True
+    mask = sel[idx[n]]
+    return oracle.coalesce(c.dims, [ix[mask] for ix in idx], vals[mask])
+
+
+def test_fullsize_amazon_mttkrp_sampled_rows(amazon):
+    B, c, X, idx, vals, F = amazon
+    layout = [X.layout(n) for n in range(3)]
+    assert any(nb > 1 for nb, _, _ in layout), layout      # the default layout blocks at least one copy
+    rng = np.random.default_rng(4)
+    Fd = [torch.from_numpy(f).cuda() for f in F]
+    for n, I in enumerate(c.dims):
+        counts = np.bincount(idx[n], minlength=I)
+        rows = np.unique(np.concatenate([rng.integers(0, I, 60), [np.argmax(counts), np.argmin(counts), 0, I - 1]]))
+        M = torch.full((I, c.R), float("nan"), dtype=torch.float64, device="cuda")
+        B.cstf_mttkrp(X, n, Fd, M)
+        torch.cuda.synchronize()
+        got = M[torch.from_numpy(rows).cuda()].cpu().numpy()
+        want = oracle.mttkrp_rows(sub_tensor(c, idx, vals, n, rows), n, F, rows)
+        assert normwise(got, want) <= TOL, (n, layout[n])
+        assert not torch.isnan(M).any().item()
+        del M
+
+
+def test_fullsize_amazon_admm_sampled_rows(amazon):
+    """The row-resident R = 64 ADMM (DMMA, row-group prefetch) on the 4.8M rows of
+    mode 1, 10 passes (eps = 0, L930-933): sampled rows vs the oracle's Alg. 2."""
+    B, c, X, idx, vals, F = amazon
+    I, R = c.dims[0], c.R
+    Fs = [oracle.normalize(f)[0] for f in F]
+    S = oracle.hadamard_except([oracle.gram(f) for f in Fs], 0)
+    M = datagen.uniform(11, 1, I * R).reshape(I, R) * 100.0 - 20.0
+    H = datagen.uniform(11, 2, I * R).reshape(I, R)
+    Hd, Ud = torch.from_numpy(H.copy()).cuda(), torch.zeros(I, R, dtype=torch.float64, device="cuda")
+    B.cstf_admm_update(torch.from_numpy(M).cuda(), torch.from_numpy(S).cuda(), Hd, Ud, tol=0.0, max_iter=10)
+    rows = np.random.default_rng(5).choice(I, 300, replace=False)
+    Hr, Ur, _ = oracle.admm(M[rows], S, H[rows], np.zeros((rows.size, R)), tol=0.0, max_iter=10)
+    torch.cuda.synchronize()
+    assert normwise(Hd[torch.from_numpy(rows).cuda()].cpu().numpy(), Hr) <= TOL
+    assert normwise(Ud[torch.from_numpy(rows).cuda()].cpu().numpy(), Ur) <= TOL

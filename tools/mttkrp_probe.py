@@ -14,7 +14,11 @@ import datagen  # noqa: E402
 from paper_conf_icpp_sohksc24_b200 import binding as B  # noqa: E402
 
 
-def timed(fn, reps=10):
+REPS = int(os.environ.get("PROBE_REPS", "10"))
+MODES = os.environ.get("PROBE_MODES")   # e.g. "1,3": only these modes
+
+
+def timed(fn, reps=REPS):
     fn()
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -43,6 +47,8 @@ def main():
     print(f"{name}: load {time.time() - t0:.1f}s", flush=True)
     F = [torch.from_numpy(f).cuda() for f in datagen.init_factors(cfg.dims, cfg.R, cfg.seed)]
     for n, I in enumerate(cfg.dims):
+        if MODES and str(n) not in MODES.split(","):
+            continue
         M = torch.empty(I, cfg.R, dtype=torch.float64, device="cuda")
         ref = None
         out = []

@@ -779,9 +779,7 @@ cstf_status launch_dmma_one(const KArgs& k, int& grid, cudaStream_t st) {
   }
   const int64_t groups = (k.I + 7) / 8;
   int64_t g = (groups + kWarpsA - 1) / kWarpsA;
-  int64_t cap = (int64_t)device_info().sms * per_sm[nsl];
-  if (const char* ge = getenv("CSTF_ADMM_CTAS_PER_SM"))            // experiment: leave SM room
-    if (atoi(ge) > 0) cap = std::min<int64_t>(cap, (int64_t)device_info().sms * atoi(ge));
+  const int64_t cap = (int64_t)device_info().sms * per_sm[nsl];
   if (g > cap) g = cap;
   grid = (int)(g < 1 ? 1 : g);
   k_admm_dmma<RP, GRAM, MU, IREG, PREF, FNN><<<grid, kThreads, smem, st>>>(k);

@@ -935,8 +935,6 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
       CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
       a.queue = w.queue.as<unsigned long long>();
       grid = std::min(grid, di.sms * mttkrp_minb(nnz, ms.Ivirt, R, false));
-      if (const char* ge = getenv("CSTF_MTTKRP_CTAS_PER_SM"))      // experiment: leave SM room
-        if (atoi(ge) > 0) grid = std::min(grid, di.sms * atoi(ge));
     }
   }
   {

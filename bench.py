@@ -41,7 +41,7 @@ from paper_conf_icpp_sohksc24_b200 import costmodel as cm  # noqa: E402
 
 METRIC = "cSTF outer-iteration time (s) and ADMM update HBM GB/s at 1/2/4/8 B200"
 PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
-FP64_PEAK_TFLOPS = 37.1      # measured on this pool's B200 (DFMA and DMMA alike), profiles/r01_microbench.txt
+FP64_PEAK_TFLOPS = 37.1      # fallback: measured on this pool's B200 (DFMA and DMMA alike), profiles/r01_microbench.txt
 L2_GATHER_GBS = 19890.0      # measured L2->SM random 256-byte row gathers, 7.4 MB tables (same microbench)
 L1_GATHER_GBS = 28855.0      # measured all-L1-hit 256-byte row gathers (16 lanes x 16 B, two 200-row tables):
                              # the on-chip ceiling of the MTTKRP access (tools/gather_probe.cu, profiles/r01_gather_probe.txt)
@@ -333,6 +333,15 @@ def main():
 
     # nvidia-smi needs a few hundred ms before its first sample: start it now, so
     # it samples the (identical) warm-up work and the timed region
+    # the ADMM roofline denominator, measured live on this box: the FP64
+    # tensor-path (DMMA) peak from the bench-only library, before the timed region
+    try:
+        from paper_conf_icpp_sohksc24_b200 import ablation as AB
+        fp64_peak, fp64_src = AB.fp64_peak(stream), ("measured live on this box: chain-only DMMA.8x8x4 kernel "
+                                                     "(cstf_ablation_fp64_peak, best of 3)")
+    except Exception as e:                   # keep the committed microbench figure
+        fp64_peak, fp64_src = FP64_PEAK_TFLOPS, (f"tools/microbench.cu -> profiles/r01_microbench.txt "
+                                                 f"(live measurement failed: {e})")
     clocks = ClockSampler(local)
     clocks.start()
     # warm-up: W outer iterations
@@ -399,14 +408,13 @@ def main():
     fl_eq3 = sum(10 * cm.admm_flops_per_row_iter(R) * I for I in cfg.dims)
     roof_admm = {"kernel": "admm (k_admm_dmma, row-resident, FNN passes)", "bound": "fp64",
                  "achieved": fl_exec / (upd_ms * 1e-3) / 1e12 if upd_ms > 0 else None,
-                 "peak": FP64_PEAK_TFLOPS, "unit": "TFLOP/s",
-                 "peak_source": "measured FP64 DMMA/DFMA peak: tools/microbench.cu -> profiles/r01_microbench.txt "
-                                "(MEASURED_PEAKS.json has no FP64 figure)",
+                 "peak": fp64_peak, "unit": "TFLOP/s",
+                 "peak_source": fp64_src + " (MEASURED_PEAKS.json has no FP64 figure)",
                  "flops": "executed: DMMA products 2 RP^2 + FNN element-wise 3R per pass + 13R last pass + "
                           "fused Gram tiles, per row (costmodel.admm_flops_executed)",
                  "eq3_flops_achieved": fl_eq3 / (upd_ms * 1e-3) / 1e12 if upd_ms > 0 else None,
                  "per_mode_ms": (mp[:, 2] / K).tolist()}
-    roof_admm["frac"] = roof_admm["achieved"] / FP64_PEAK_TFLOPS if upd_ms > 0 else None
+    roof_admm["frac"] = roof_admm["achieved"] / fp64_peak if upd_ms > 0 else None
     if traffic and "admm" in traffic:
         ta = traffic["admm"]
         roof_admm["ncu_fp64_datapath_frac"] = ta.get("fp64_datapath_frac")

@@ -43,6 +43,13 @@ int cstf_ablation_admm(int arm, const double* d_M, const double* d_S, double* d_
 const char* cstf_ablation_last_error(void);
 /* kernel launches + cuBLAS calls issued by the last cstf_ablation_admm call */
 int64_t cstf_ablation_last_calls(void);
+/* Measured FP64 tensor-path peak of the current device in TFLOP/s: best of 3
+ * launches of a chain-only mma.sync.m8n8k4.f64 kernel (SASS DMMA.8x8x4; 8
+ * independent accumulators per warp, 8 CTAs of 256 threads per SM, ~10 ms each)
+ * on `stream`, after a warm-up launch.  The roofline denominator of the ADMM
+ * (SURVEY s8(d)).  Blocking; allocates and frees a small buffer.  Returns a
+ * negative value on any CUDA error. */
+double cstf_ablation_fp64_peak(void* stream);
 
 #ifdef __cplusplus
 }

@@ -18,6 +18,8 @@ _lib.cstf_ablation_admm.argtypes = [ctypes.c_int, ctypes.c_void_p, ctypes.c_void
                                     ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p]
 _lib.cstf_ablation_last_error.restype = ctypes.c_char_p
 _lib.cstf_ablation_last_calls.restype = ctypes.c_int64
+_lib.cstf_ablation_fp64_peak.restype = ctypes.c_double
+_lib.cstf_ablation_fp64_peak.argtypes = [ctypes.c_void_p]
 
 BASELINE, OF, PI, OF_PI = 0, 1, 2, 3
 ARMS = {"baseline": BASELINE, "of": OF, "pi": PI, "of_pi": OF_PI}
@@ -38,3 +40,13 @@ def admm(arm: int, M, S, H, U, max_iter: int = 10, stream=None) -> dict:
         raise RuntimeError("cstf_ablation_admm: " + _lib.cstf_ablation_last_error().decode())
     return dict(iters=int(st[0]), rho=st[1], r_primal=st[2], s_dual=st[3], normH2=st[4], normU2=st[5],
                 calls=int(_lib.cstf_ablation_last_calls()))
+
+
+def fp64_peak(stream=None) -> float:
+    """Measured FP64 DMMA peak of the current device (TFLOP/s), cstf_ablation_fp64_peak."""
+    import torch
+    st = stream if stream is not None else torch.cuda.current_stream()
+    v = float(_lib.cstf_ablation_fp64_peak(ctypes.c_void_p(st.cuda_stream)))
+    if v <= 0:
+        raise RuntimeError("cstf_ablation_fp64_peak failed")
+    return v

@@ -242,6 +242,25 @@ int ensure(Ws& w, size_t bytes) {
   return 0;
 }
 
+// FP64 tensor-path peak ("measure on the box the FP64 DMMA peak"):
+// 8 independent m8n8k4 f64 accumulator chains per warp, no memory traffic.
+__global__ void __launch_bounds__(256) k_dmma_peak(double* out, int iters) {
+  const double a = threadIdx.x * 1e-3, b = threadIdx.x * 2e-3;
+  double c[8][2];
+#pragma unroll
+  for (int t = 0; t < 8; t++) c[t][0] = c[t][1] = 0.0;
+  for (int i = 0; i < iters; i++) {
+#pragma unroll
+    for (int t = 0; t < 8; t++)
+      asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+                   : "+d"(c[t][0]), "+d"(c[t][1]) : "d"(a), "d"(b));
+  }
+  double s = 0.0;
+#pragma unroll
+  for (int t = 0; t < 8; t++) s += c[t][0] + c[t][1];
+  out[blockIdx.x * blockDim.x + threadIdx.x] = s;
+}
+
 }  // namespace
 
 extern "C" {
@@ -334,6 +353,37 @@ int cstf_ablation_admm(int arm, const double* d_M, const double* d_S, double* d_
   if (stats_out)
     for (int k = 0; k < 6; k++) stats_out[k] = host[k];
   return 0;
+}
+
+double cstf_ablation_fp64_peak(void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  int dev = 0, sms = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+    return -1.0;
+  const int grid = sms * 8, bs = 256, iters = 4096;
+  double* out = nullptr;
+  cudaEvent_t e0, e1;
+  if (cudaMalloc(&out, (size_t)grid * bs * 8) != cudaSuccess) return -1.0;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  k_dmma_peak<<<grid, bs, 0, st>>>(out, 64);                 // warm-up (clocks up)
+  float best = 1e30f;
+  for (int r = 0; r < 3; r++) {
+    cudaEventRecord(e0, st);
+    k_dmma_peak<<<grid, bs, 0, st>>>(out, iters);
+    cudaEventRecord(e1, st);
+    cudaEventSynchronize(e1);
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    best = std::min(best, ms);
+  }
+  const cudaError_t e = cudaGetLastError();
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaFree(out);
+  if (e != cudaSuccess || best <= 0.f) return -1.0;
+  const double flops = 2.0 * 256 * 8 * (double)iters * grid * (bs / 32);    // 8 chains x 512 flops per warp
+  return flops / (best * 1e-3) / 1e12;
 }
 
 }  // extern "C"

@@ -53,3 +53,15 @@ def test_ablation_arm_matches_oracle(A, arm, I, R, max_iter):
     # the arms issue the call shape they claim: per pass 7 (baseline), 4 (OF), 6 (PI), 3 (OF+PI)
     per_pass = {"baseline": 8, "of": 4, "pi": 7, "of_pi": 3}[arm]
     assert st["calls"] >= per_pass * max_iter
+
+
+def test_fp64_peak_microbench():
+    """The live FP64 DMMA peak the bench divides by: B200 runs 128 FP64
+    flops per clock and SM on the tensor path (148 SMs x 1.965 GHz = 37.2 TF/s); a
+    power-capped clock lowers it, nothing raises it above the clock-scaled bound."""
+    import torch
+    from paper_conf_icpp_sohksc24_b200 import ablation as AB
+    v = AB.fp64_peak()
+    p = torch.cuda.get_device_properties(0)
+    bound = p.multi_processor_count * 128 * 1.965e9 / 1e12 * 1.02
+    assert 0.3 * bound < v <= bound, (v, bound)

@@ -146,7 +146,8 @@ def test_ablation_library_exports():
     so = ctypes.CDLL(path)
     txt = re.sub(r"/\*.*?\*/", "", open(os.path.join(ROOT, "include", "cstf_ablation.h")).read(), flags=re.S)
     syms = set(re.findall(r"\b(cstf_[a-z_0-9]+)\s*\(", txt))
-    assert syms == {"cstf_ablation_admm", "cstf_ablation_last_error", "cstf_ablation_last_calls"}
+    assert syms == {"cstf_ablation_admm", "cstf_ablation_last_error", "cstf_ablation_last_calls",
+                    "cstf_ablation_fp64_peak"}
     for s in syms:
         assert hasattr(so, s)
     so.cstf_ablation_admm.restype = ctypes.c_int

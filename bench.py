@@ -123,6 +123,9 @@ class ClockSampler:
 def oracle_outer_iteration(cfg, idx, vals, R, steps, warmup):
     """The FP64 oracle as it stands: one outer iteration (eps = 0, 10 inner) per step."""
     import oracle
+    # all host cores of this process (torchrun sets OMP_NUM_THREADS=1 in every rank;
+    # only rank 0 runs the oracle); the count reported is the one in effect
+    cores = oracle.set_threads(len(os.sched_getaffinity(0)))
     t0 = time.time()
     X = oracle.coalesce(cfg.dims, idx, vals)
     t_coalesce = time.time() - t0
@@ -134,7 +137,6 @@ def oracle_outer_iteration(cfg, idx, vals, R, steps, warmup):
         dt = time.perf_counter() - t0
         if s >= warmup:
             times.append(dt)
-    cores = len(os.sched_getaffinity(0))
     return float(np.mean(times)), cores, t_coalesce
 
 

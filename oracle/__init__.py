@@ -62,10 +62,24 @@ def _get():
         L.oracle_mu.argtypes = [i64, i32, p, p, p, i32]
         L.oracle_fit.restype = d
         L.oracle_fit.argtypes = [i32, i32, d, i64, p, p, p, p]
+        L.oracle_set_threads.argtypes = [i32]
+        L.oracle_threads.restype = i32
         L.oracle_factorize.argtypes = [i32, p, i64, p, p, d, i32, i32, d, d, i32, d, i32, i32, i32, d, i32,
                                        p, p, p, p, p, p, p]
         _lib = L
     return _lib
+
+
+def set_threads(n: int) -> int:
+    """OpenMP threads of the oracle's parallel regions (results do not depend on it,
+    pin P11); returns the count now in effect."""
+    L = _get()
+    L.oracle_set_threads(int(n))
+    return int(L.oracle_threads())
+
+
+def threads() -> int:
+    return int(_get().oracle_threads())
 
 
 def _ptrs(arrays, ctype=ctypes.c_void_p):

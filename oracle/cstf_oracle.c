@@ -57,6 +57,12 @@ static double prox_apply(int prox, double x, double tau) {
   }
 }
 
+/* Thread count of the OpenMP regions (infrastructure, no arithmetic): torchrun sets
+ * OMP_NUM_THREADS=1 in every rank, so the bench's rank 0 sets the count it reports. */
+#include <omp.h>
+void oracle_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
+int oracle_threads(void) { return omp_get_max_threads(); }
+
 static double now_ms(void) {
   struct timespec ts; clock_gettime(CLOCK_MONOTONIC, &ts);
   return ts.tv_sec * 1e3 + ts.tv_nsec * 1e-6;

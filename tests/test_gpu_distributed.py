@@ -23,7 +23,7 @@ torch.cuda.set_device(0)
 rank, P = dist.get_rank(), dist.get_world_size()
 comm = B.cstf_comm_create_nccl() if COMM == "nccl" else B.cstf_comm_create_host()
 cfg, scale, R, tol, outer = CASE
-c = datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
+c = datagen.CONFIGS[cfg] if scale == 0 else datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
 idx, vals = c.generate()
 X = B.cstf_tensor_load_coo(c.dims, idx, vals, comm=comm)
 start = datagen.init_factors(c.dims, R, c.seed)
@@ -37,6 +37,7 @@ assert np.array_equal(rep["fit"], rep2["fit"]), (rep["fit"], rep2["fit"])
 out = {"fit": rep["fit"].tolist(), "iters": rep["iters"].tolist(), "comm_ms": rep["phase_ms"]["COMM"],
        "nblk": [X.layout(n)[0] for n in range(len(c.dims))]}
 if rank == 0:
+    oracle.set_threads(len(os.sched_getaffinity(0)))    # torchrun runs every rank with OMP_NUM_THREADS=1
     ref = oracle.coalesce(c.dims, idx, vals)
     orc = oracle.factorize(ref, start, outer_iters=outer, tol=tol, max_iter=10)
     ncmp, tie = compare_iteration_counts(rep["iters"], orc, tol if tol > 0 else 1e-2)
@@ -80,6 +81,10 @@ def run(tmp_path, nproc, case, port, comm="host"):
     (3, ("enron", 60, 16, 1e-2, 5), 29619, "blk"),
     (2, ("delicious", 1000, 32, 0.0, 3), 29620, "hot"),   # hot-row tables over internal labels (forced)
     (3, ("delicious", 1000, 16, 1e-2, 4), 29622, "hot"),
+    # full size (scale 0), the bench protocol (eps = 0, 10 passes, one outer iteration):
+    # configs[2] Enron-shaped (54M nonzeros) and configs[3] Delicious-shaped (140M) on 2 ranks
+    (2, ("enron", 0, 32, 0.0, 1), 29623, "1"),
+    (2, ("delicious", 0, 32, 0.0, 1), 29624, "1"),
 ])
 def test_partitioned_factorize_matches_oracle(tmp_path, nproc, case, port, peer, monkeypatch):
     """peer: CSTF_PEER_STORE for the host communicator, or "nccl" (one rank: the
@@ -151,7 +156,7 @@ def test_loopback_threads_match_oracle(nparts, cfg, scale, R, tol):
     import oracle
     from parity_util import compare_iteration_counts
     from paper_conf_icpp_sohksc24_b200 import binding as B
-    c = datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
+    c = datagen.CONFIGS[cfg] if scale == 0 else datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
     out, idx, vals, start = _loopback_run(B, torch, nparts, c, R, tol, 4)
     assert all(o[0] == "ok" for o in out), out
     ref = oracle.coalesce(c.dims, idx, vals)
@@ -194,10 +199,12 @@ dist.init_process_group("gloo")
 torch.cuda.set_device(0)
 rank, P = dist.get_rank(), dist.get_world_size()
 comm = B.cstf_comm_create_host()
+if rank == 0:
+    oracle.set_threads(len(os.sched_getaffinity(0)))    # torchrun runs every rank with OMP_NUM_THREADS=1
 res = []
 # small -> larger (replica buffer re-allocated, peer mappings refreshed) -> small again
 for cfg, scale, R in (("nell2", 80, 16), ("enron", 30, 32), ("nell2", 80, 16), ("nell2", 40, 32)):
-    c = datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
+    c = datagen.CONFIGS[cfg] if scale == 0 else datagen.CONFIGS[cfg].scaled(scale, nnz_factor=scale * 20)
     idx, vals = c.generate()
     X = B.cstf_tensor_load_coo(c.dims, idx, vals, comm=comm)
     start = datagen.init_factors(c.dims, R, 3)

@@ -33,15 +33,32 @@ constexpr int kWarps = 8;  // per CTA
 // warps), < 64 -> 3 for R = 32 / 64 (80 registers; Delicious mode 2, 56 per row:
 // 10.81 -> 10.0 ms), else 2 (long rows).  Virtual rows of L2-blocked copies (`tiled`)
 // keep 4 below 64 (Amazon, ~20 per virtual row: 531 -> 592 ms with 3).
-// CSTF_MTTKRP_MINB=2/3/4 forces (experiments).
-int mttkrp_minb(int64_t nnz, int64_t rows, int R, bool tiled) {
+// Hot-row copies at R = 32 (factors streamed from HBM) trade warps for gathers in
+// flight per warp (mttkrp_unr): short rows 3 CTAs with 2 steps of row loads issued
+// together, medium rows 2 CTAs with 4 steps (bench path, Delicious modes 1 / 2:
+// 11.84 -> 11.26 ms, 9.90 -> 9.44 ms; tools/bench_variants.sh,
+// profiles/r02_mttkrp_unroll_variants.txt).
+// CSTF_MTTKRP_MINB=2/3/4 and CSTF_MTTKRP_UNR=1..4 force (experiments).
+int mttkrp_minb(int64_t nnz, int64_t rows, int R, bool tiled, bool hot = false, int nother = 3) {
   if (const char* e = getenv("CSTF_MTTKRP_MINB")) {
     const int v = atoi(e);
     if (v == 2 || v == 4 || (v == 3 && (R == 32 || R == 64))) return v;
   }
+  if (hot && R == 32 && !tiled && nother <= 4 && nnz < 64 * rows) return nnz < 16 * rows ? 3 : 2;
   if (nnz < 16 * rows) return 4;
   if (nnz < 64 * rows) return (!tiled && (R == 32 || R == 64)) ? 3 : 4;
   return 2;
+}
+
+// Steps of row gathers issued before the first product (hot-row copies, R = 32; 1 elsewhere)
+int mttkrp_unr(int64_t nnz, int64_t rows, int R, bool tiled, bool hot, int nother = 3) {
+  if (!hot || R != 32 || nother > 4) return 1;
+  if (const char* e = getenv("CSTF_MTTKRP_UNR")) {
+    const int v = atoi(e);
+    if (v >= 1 && v <= 4) return v;
+  }
+  if (tiled || nnz >= 64 * rows) return 1;
+  return nnz < 16 * rows ? 2 : 4;
 }
 
 struct MArgs {
@@ -113,7 +130,7 @@ __device__ __forceinline__ const double2* row_addr(const char* base, unsigned j)
 // One warp processes chunk c.  Fb[q] = lane's byte offset into the row source of
 // slot q (a factor in global memory, or the shared-memory slab of a k-blocked
 // copy, already shifted by the slab's first row).
-template <int NOTHER, int R, int RECB, int GL = 0, bool HOT = false>
+template <int NOTHER, int R, int RECB, int GL = 0, bool HOT = false, int UNR = 1>
 __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const char* const* Fb, int4* srec,
                                               const char* const* HFb = nullptr) {
   constexpr int RV = R / 2;                    // double2 per row
@@ -182,6 +199,50 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
           continue;
         }
         const int run = (int)min((int64_t)(nb - t), seg_end - p);
+        if constexpr (UNR > 1) {
+          // UNR steps per iteration, every row load of all of them issued before the
+          // first product: UNR x NOTHER gathers in flight per lane instead of NOTHER
+          for (int done = 0; done < run; done += UNR * P) {
+            double2 xs[UNR][NOTHER][VPL];
+            double vv[UNR];
+#pragma unroll
+            for (int u = 0; u < UNR; u++) {
+              const int d = done + u * P;
+              const bool ok = (d + sg) < run;
+              const int src = ok ? t + d + sg : t + done;
+              unsigned w[NW];
+#pragma unroll
+              for (int k = 0; k < NV; k++) {
+                const int4 x = sr[src * NV + k];
+                w[4 * k] = x.x; w[4 * k + 1] = x.y; w[4 * k + 2] = x.z; w[4 * k + 3] = x.w;
+              }
+              vv[u] = ok ? __hiloint2double((int)w[NW - 1], (int)w[NW - 2]) : 0.0;
+#pragma unroll
+              for (int qq = 0; qq < NOTHER; qq++) {
+                const char* base = Fb[qq];
+                unsigned j = w[qq];
+                if constexpr (HOT) {
+                  if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
+                }
+                const double2* rp = row_addr<ROWB>(base, j);
+#pragma unroll
+                for (int s = 0; s < VPL; s++) xs[u][qq][s] = rp[s * G];
+              }
+            }
+#pragma unroll
+            for (int u = 0; u < UNR; u++)
+#pragma unroll
+              for (int s = 0; s < VPL; s++) {
+                double2 f = xs[u][0][s];
+#pragma unroll
+                for (int qq = 1; qq < NOTHER; qq++) { f.x *= xs[u][qq][s].x; f.y *= xs[u][qq][s].y; }
+                acc[s].x = fma(vv[u], f.x, acc[s].x);
+                acc[s].y = fma(vv[u], f.y, acc[s].y);
+              }
+          }
+          t += run;
+          continue;
+        }
 #pragma unroll 4
         for (int done = 0; done < run; done += P) {
           const bool ok = (done + sg) < run;
@@ -226,7 +287,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
 }
 
 // MINB: CTAs per SM the register budget targets (2 for long rows, 4 for short ones)
-template <int NOTHER, int R, int RECB, int MINB, int GL = 0, bool HOT = false>
+template <int NOTHER, int R, int RECB, int MINB, int GL = 0, bool HOT = false, int UNR = 1>
 __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
   constexpr int G = GL ? GL : ((R / 2) < 32 ? (R / 2) : 32);
   const int gl = (threadIdx.x & 31) % G;
@@ -251,11 +312,11 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
       if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
       c = __shfl_sync(0xffffffffu, c, 0);
       if ((int64_t)c >= a.nchunks) break;
-      process_chunk<NOTHER, R, RECB, GL, HOT>(a, (int64_t)c, Fb, srec, HFb);
+      process_chunk<NOTHER, R, RECB, GL, HOT, UNR>(a, (int64_t)c, Fb, srec, HFb);
     }
     return;
   }
-  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT>(a, c, Fb, srec, HFb);
+  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT, UNR>(a, c, Fb, srec, HFb);
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -428,7 +489,7 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
   // CTAs per SM by nonzeros per row (mttkrp_minb): short rows -- row flushes dominate,
   // latency hiding needs warps -- 4 (64 registers); medium rows (R = 32 / 64) 3 (80);
   // long rows 2 (128)
-  const int minb = mttkrp_minb(a.nnz, a.I - a.rbase, a.R, a.l2blocked != 0);
+  const int minb = mttkrp_minb(a.nnz, a.I - a.rbase, a.R, a.l2blocked != 0, hot, NOTHER);
   const bool short_rows = minb == 4;
   const bool mid_rows = minb == 3;
   if (tiled) {
@@ -449,6 +510,19 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
   }
   GCASE(32, 8) GCASE(64, 16)
 #undef GCASE
+  // hot-row copies at R = 32: unrolled gathers (mttkrp_unr; 5+ other modes would spill)
+  if constexpr (NOTHER <= 4) {
+    const int unr = (hot && a.R == 32) ? mttkrp_unr(a.nnz, a.I - a.rbase, a.R, a.l2blocked != 0, hot, NOTHER) : 1;
+#define UCASE(UU)                                                                                      \
+  if (unr == UU) {                                                                                     \
+    if (short_rows) k_mttkrp_fast<NOTHER, 32, RECB, 4, 0, true, UU><<<grid, kWarps * 32, 0, st>>>(a);   \
+    else if (mid_rows) k_mttkrp_fast<NOTHER, 32, RECB, 3, 0, true, UU><<<grid, kWarps * 32, 0, st>>>(a); \
+    else k_mttkrp_fast<NOTHER, 32, RECB, 2, 0, true, UU><<<grid, kWarps * 32, 0, st>>>(a);              \
+    return true;                                                                                       \
+  }
+    UCASE(2) UCASE(3) UCASE(4)
+#undef UCASE
+  }
   if (hot) {           // copies with hot-row slots (large factors): R = 16 / 32 / 64, else generic
     switch (a.R) {
 #define HCASE(RR)                                                                              \
@@ -599,7 +673,7 @@ cstf_status mttkrp_l2_blocked(const ModeStore& ms, MArgs& a, int R, int gl, doub
     if (B == 1) return fail(CSTF_ERR_OUT_OF_MEMORY, "MTTKRP partial rows of one L2 block (set CSTF_L2_BLOCK=0)");
     B = (B + 1) / 2;
   }
-  const int ctas = di.sms * mttkrp_minb(nnz, ms.Ivirt, R, true);   // resident CTAs only (= launch_fast's budget)
+  const int ctas = di.sms * mttkrp_minb(nnz, ms.Ivirt, R, true, hot, a.nother);   // resident CTAs only (= launch_fast's budget)
   a.l2blocked = 1;
   // chunk: the window in flight (resident warps x chunk) about half a block
   int64_t chunk = (nnz / std::max<int64_t>(nblk, 1)) / (2 * (int64_t)ctas * kWarps);
@@ -934,7 +1008,7 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
       CSTF_TRY(w.queue.ensure(8));
       CSTF_CUDA(cudaMemsetAsync(w.queue.p, 0, 8, st));
       a.queue = w.queue.as<unsigned long long>();
-      grid = std::min(grid, di.sms * mttkrp_minb(nnz, ms.Ivirt, R, false));
+      grid = std::min(grid, di.sms * mttkrp_minb(nnz, ms.Ivirt, R, false, hot, N - 1));
     }
   }
   {

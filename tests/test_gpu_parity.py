@@ -723,6 +723,32 @@ def test_mttkrp_hot_row_tables(B, R, window, monkeypatch):
     assert normwise(host(M), oracle.mttkrp(ref, 0, F2)) <= TOL
 
 
+@pytest.mark.parametrize("unr", ["1", "2", "3", "4"])
+def test_mttkrp_hot_unrolled_gathers(B, unr, monkeypatch):
+    """Hot-row copies at R = 32 issue the row loads of several steps before the first
+    product (mttkrp_unr: 2 steps for short rows, 4 for medium ones).  Forced hot rows,
+    one mode per row class (long 3333 / short 10 / medium 37 / long 7500 nonzeros per
+    row): every unroll depth matches the oracle, and -- the per-group accumulation
+    order is unchanged -- is bitwise equal to the one-step kernel."""
+    monkeypatch.setenv("CSTF_HOT_ROWS", "400")
+    dims = (90, 30000, 8000, 40)
+    idx, vals = datagen.coo(dims, (2, 2, 3, 1), 300_000, 52)
+    X = B.cstf_tensor_load_coo(dims, idx, vals)
+    ref = oracle.coalesce(dims, idx, vals)
+    F = datagen.init_factors(dims, 32, 10)
+    Fd = [cu(f) for f in F]
+    for n in range(4):
+        monkeypatch.setenv("CSTF_MTTKRP_UNR", "1")
+        M1 = cu(np.full((dims[n], 32), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M1)
+        monkeypatch.setenv("CSTF_MTTKRP_UNR", unr)
+        M = cu(np.full((dims[n], 32), np.nan))
+        B.cstf_mttkrp(X, n, Fd, M)
+        got = host(M).copy()
+        assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, n
+        assert np.array_equal(got, host(M1)), n
+
+
 @pytest.mark.parametrize("tol,R", [(1e-2, 16), (0.0, 32)])
 def test_factorize_hot_row_tables(B, tol, R, monkeypatch):
     """factorize keeps the hot-row tables current after every update (forced hot rows)."""

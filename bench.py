@@ -65,7 +65,8 @@ def measured_traffic(workload):
             d = json.load(f)
         t = d.get(workload)
         if t is not None:
-            t = dict(t, source=d.get("source", "profiles/r02_traffic.json"))
+            t = dict(t, source="profiles/r02_traffic.json (ncu capture of " + d.get("source", "?") + "; " +
+                     d.get("how", "") + ")")
         return t
     except Exception:
         return None

@@ -92,6 +92,7 @@ _decl("cstf_tensor_info", c_int, [c_void_p, ctypes.POINTER(c_int), c_void_p, cty
 _decl("cstf_tensor_export_coo", c_int, [c_void_p, c_void_p, c_void_p])
 _decl("cstf_tensor_layout", c_int, [c_void_p, c_int, ctypes.POINTER(c_int64), ctypes.POINTER(c_int64),
                                     ctypes.POINTER(c_int)])
+_decl("cstf_tensor_record_bytes", c_int, [c_void_p, c_int, ctypes.POINTER(c_int)])
 _decl("cstf_tensor_free", None, [c_void_p])
 _decl("cstf_mttkrp", c_int, [c_void_p, c_int, c_int, c_void_p, c_void_p, c_void_p])
 _decl("cstf_gram", c_int, [c_void_p, c_int64, c_int, c_void_p, c_void_p, c_void_p])
@@ -108,7 +109,7 @@ _decl("cstf_factorize_host", c_int, [c_void_p, ctypes.POINTER(Opts), c_void_p, c
 EXPORTED = ["cstf_status_string", "cstf_last_error_message", "cstf_version", "cstf_get_unique_id",
             "cstf_comm_create", "cstf_comm_create_host", "cstf_comm_loopback", "cstf_comm_info", "cstf_comm_destroy",
             "cstf_partition_rows",
-            "cstf_tensor_load_coo", "cstf_tensor_info", "cstf_tensor_layout", "cstf_tensor_export_coo", "cstf_tensor_free",
+            "cstf_tensor_load_coo", "cstf_tensor_info", "cstf_tensor_layout", "cstf_tensor_record_bytes", "cstf_tensor_export_coo", "cstf_tensor_free",
             "cstf_mttkrp", "cstf_gram", "cstf_normalize", "cstf_admm_update", "cstf_hals_update",
             "cstf_mu_update", "cstf_factorize",
             "cstf_factorize_host", "cstf_kernel_launch_count", "cstf_release_workspace"]
@@ -276,6 +277,12 @@ class Tensor:
         _check(_lib.cstf_tensor_layout(self.handle, mode, ctypes.byref(nb), ctypes.byref(br), ctypes.byref(bm)),
                "cstf_tensor_layout")
         return nb.value, br.value, bm.value
+
+    def record_bytes(self, mode: int) -> int:
+        """Bytes per nonzero record of the mode copy (16 = packed 4-mode records)."""
+        rb = c_int()
+        _check(_lib.cstf_tensor_record_bytes(self.handle, mode, ctypes.byref(rb)), "cstf_tensor_record_bytes")
+        return rb.value
 
     def export_coo(self):
         info = self.info()

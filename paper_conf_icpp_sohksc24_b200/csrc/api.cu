@@ -597,6 +597,12 @@ cstf_status cstf_tensor_layout(const cstf_tensor* X, int mode, int64_t* nblk, in
   return CSTF_OK;
 }
 
+cstf_status cstf_tensor_record_bytes(const cstf_tensor* X, int mode, int* record_bytes) {
+  if (!X || !record_bytes || mode < 0 || mode >= X->N) return fail(CSTF_ERR_INVALID_ARG, "tensor is NULL or bad mode");
+  *record_bytes = X->mode[mode].recb;
+  return CSTF_OK;
+}
+
 cstf_status cstf_tensor_export_coo(const cstf_tensor* X, int32_t* const* host_idx, double* host_vals) {
   if (!X || (X->nnz > 0 && (!host_idx || !host_vals))) return fail(CSTF_ERR_INVALID_ARG, "export arguments");
   if (X->partitioned) return fail(CSTF_ERR_UNSUPPORTED, "export of a partitioned tensor");

@@ -116,6 +116,15 @@ struct ModeStore {
   // hot-row tables: bit q set = the records of slot q name hot rows of factor other[q]
   // by (0x80000000 | hot slot)
   int hotmask = 0;
+  // Packed 16-byte records (round 2): when the row indices of
+  // the N-1 = 3 gathered slots fit one 64-bit word, record = {uint64 key, f64 x} with
+  // slot q at bits [pk_sh[q], pk_sh[q] + width) of key: the row, or pk_hot[q] | hot slot
+  // (pk_hot[q] = the field's top bit, 0 for slots without hot rows).  Not for L2-blocked
+  // copies.  CSTF_PACK=0 keeps the 32-byte records.
+  bool pk = false;
+  int pk_sh[7] = {0};
+  uint32_t pk_mask[7] = {0};
+  uint32_t pk_hot[7] = {0};
 };
 inline int record_bytes(int N) { return ((4 * (N - 1) + 8) + 15) / 16 * 16; }
 

@@ -80,7 +80,41 @@ struct MArgs {
   unsigned long long* queue;  // dynamic chunk counter (L2-blocked copies) or null = static grid stride
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
   int l2blocked;        // launch over an L2-blocked copy (rows are virtual rows)
+  int pk;               // packed 16-byte records (ModeStore::pk): slot q = (key >> pk_sh[q]) & pk_mask[q]
+  int pk_sh[3];
+  uint32_t pk_mask[3], pk_hot[3];
 };
+
+// Field of record slot q of a packed record (key = words w0, w1): the row, or the hot
+// flag pk_hot[q] | hot slot
+__device__ __forceinline__ unsigned pk_field(const MArgs& a, int q, unsigned w0, unsigned w1) {
+  return q == 0 ? (w0 & a.pk_mask[0])
+                : (unsigned)((((unsigned long long)w1 << 32) | w0) >> a.pk_sh[q]) & a.pk_mask[q];
+}
+
+// Row source and row of slot q: the hot-row table for a hot slot, else the factor.  Both
+// record kinds resolve by selects (no branch, so the gathers of a step issue together).
+template <bool PK, bool HOT>
+__device__ __forceinline__ void slot_row(const MArgs& a, int q, const unsigned* w, const char* fb, const char* hfb,
+                                         const char*& base, unsigned& j) {
+  if constexpr (PK) {
+    const unsigned f = pk_field(a, q, w[0], w[1]);
+    if constexpr (HOT) {
+      const unsigned hb = f & a.pk_hot[q];
+      j = f ^ hb;
+      base = hb ? hfb : fb;
+    } else {
+      j = f;
+      base = fb;
+    }
+  } else {
+    j = w[q];
+    base = fb;
+    if constexpr (HOT) {            // hot row: its copy in the persisting hot-row table
+      if ((int)j < 0) { base = hfb; j &= 0x7fffffffu; }
+    }
+  }
+}
 
 // Chunks sit on the absolute grid of multiples of `chunk`, clipped to the launch's
 // nonzero range: a launch over a batch of L2 blocks splits every row exactly where
@@ -139,6 +173,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
   constexpr int P = 32 / G;                    // nonzeros per warp step
   constexpr unsigned ROWB = R * 8;
   constexpr int NW = RECB / 4;                 // 32-bit words per record
+  constexpr bool PK = RECB == 16 && NOTHER >= 3;   // packed records (3 slots in one 64-bit key)
   const int lane = threadIdx.x & 31;
   const int sg = lane / G, gl = lane % G;
   {
@@ -219,11 +254,9 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
               vv[u] = ok ? __hiloint2double((int)w[NW - 1], (int)w[NW - 2]) : 0.0;
 #pragma unroll
               for (int qq = 0; qq < NOTHER; qq++) {
-                const char* base = Fb[qq];
-                unsigned j = w[qq];
-                if constexpr (HOT) {
-                  if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
-                }
+                const char* base;
+                unsigned j;
+                slot_row<PK, HOT>(a, qq, w, Fb[qq], HOT ? HFb[qq] : nullptr, base, j);
                 const double2* rp = row_addr<ROWB>(base, j);
 #pragma unroll
                 for (int s = 0; s < VPL; s++) xs[u][qq][s] = rp[s * G];
@@ -257,11 +290,9 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
           double2 f[VPL];
 #pragma unroll
           for (int qq = 0; qq < NOTHER; qq++) {
-            const char* base = Fb[qq];
-            unsigned j = w[qq];
-            if constexpr (HOT) {            // hot row: its copy in the persisting hot-row table
-              if ((int)j < 0) { base = HFb[qq]; j &= 0x7fffffffu; }
-            }
+            const char* base;
+            unsigned j;
+            slot_row<PK, HOT>(a, qq, w, Fb[qq], HOT ? HFb[qq] : nullptr, base, j);
             const double2* rp = row_addr<ROWB>(base, j);
 #pragma unroll
             for (int s = 0; s < VPL; s++) {
@@ -373,7 +404,14 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
         for (int q = 0; q < a.nother; q++) {
           unsigned j = reinterpret_cast<const unsigned*>(r)[q];
           const double* fq = a.F[q];
-          if ((int)j < 0) { fq = a.HF[q]; j &= 0x7fffffffu; }     // hot row (hot-row table)
+          if (a.pk) {
+            const unsigned f = pk_field(a, q, reinterpret_cast<const unsigned*>(r)[0], reinterpret_cast<const unsigned*>(r)[1]);
+            j = f & ~a.pk_hot[q];
+            if (f & a.pk_hot[q]) fq = a.HF[q];
+          } else if ((int)j < 0) {
+            fq = a.HF[q];                   // hot row (hot-row table)
+            j &= 0x7fffffffu;
+          }
           const double* src = fq + (size_t)j * (unsigned)R;
 #pragma unroll
           for (int s = 0; s < CPL; s++) {
@@ -563,7 +601,7 @@ cstf_status launch_main(const MArgs& a, int grid, int tgrid, cudaStream_t st, in
   switch (a.nother) {
     case 1: done = launch_fast<1, 16>(a, grid, st, false, gl, hot); break;
     case 2: done = launch_fast<2, 16>(a, g, st, tl, gl, hot); break;
-    case 3: done = launch_fast<3, 32>(a, g, st, tl, gl, hot); break;
+    case 3: done = a.pk ? launch_fast<3, 16>(a, g, st, tl, gl, hot) : launch_fast<3, 32>(a, g, st, tl, gl, hot); break;
     case 4: done = launch_fast<4, 32>(a, g, st, tl, gl, hot); break;
     case 5: done = launch_fast<5, 32>(a, g, st, tl, gl, hot); break;
     case 6: done = launch_fast<6, 32>(a, g, st, tl, gl, hot); break;
@@ -879,6 +917,8 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.rowptr = ms.rowptr.as<int64_t>();
   a.rec = ms.rec.as<char>();
   a.recb = ms.recb;
+  a.pk = ms.pk ? 1 : 0;
+  for (int q = 0; q < 3; q++) { a.pk_sh[q] = ms.pk_sh[q]; a.pk_mask[q] = ms.pk_mask[q]; a.pk_hot[q] = ms.pk_hot[q]; }
   a.nother = N - 1;
   for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
   a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor

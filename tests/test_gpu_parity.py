@@ -212,6 +212,27 @@ def test_gram_and_normalize(B, I, R):
     assert normwise(host(G2), oracle.gram(Hn)) <= 1e-12
 
 
+@pytest.mark.parametrize("R", [32, 7])
+def test_normalize_division_exact(B, R):
+    """The column scaling divides by lambda through the rounded reciprocal plus one fma
+    correction (dense.cu div_by): bit for bit IEEE x / lambda, checked against numpy's
+    division with the returned lambda on values spread over 2^-60 .. 2^60 (plus zeros,
+    negatives and a zero column), for the paired (even R) and scalar kernels."""
+    I = 200_003
+    H = datagen.uniform(6, 78, I * R).reshape(I, R) - 0.3
+    H *= np.exp2(np.floor(datagen.uniform(6, 79, I * R) * 120.0 - 60.0)).reshape(I, R)
+    H[::97, 1] = 0.0
+    H[:, R - 1] = 0.0
+    Hd = cu(H)
+    lam = cu(np.zeros(R))
+    B.cstf_normalize(Hd, lam, cu(np.zeros((R, R))))
+    l = host(lam)
+    want = H.copy()
+    nz = l > 0
+    want[:, nz] = H[:, nz] / l[nz]
+    assert np.array_equal(host(Hd), want)
+
+
 def admm_inputs(I, R, seed, nmodes=3):
     """M, S, H, U shaped like a real update: S = Hadamard of Grams of normalised factors."""
     Fs = [oracle.normalize(datagen.uniform(seed, 10 + k, 200 * R).reshape(200, R))[0] for k in range(nmodes)]

@@ -3,7 +3,8 @@ synccheck, initcheck):
     compute-sanitizer --tool memcheck python tools/sanitize_cases.py
 Cases: the planted configs[0] factorisation (ADMM tolerance mode: speculative chunks
 + replay), the fixed-iteration protocol (fused Gram epilogue, FNN passes), forced
-L2-blocked MTTKRP (one-block batches, persisting window), forced hot-row tables, the
+L2-blocked MTTKRP (one-block batches, persisting window), forced hot-row tables, packed
+16-byte records (fast and generic kernels, export), the
 R = 64 ADMM with the cp.async row-group prefetch over several groups per warp, HALS /
 MU, and the bench-only ablation arms.  Sizes are small: the tools slow kernels 10-100x."""
 import os
@@ -24,7 +25,8 @@ def cu(a):
 
 def main():
     torch.cuda.set_device(0)
-    which = sys.argv[1:] or ["planted", "fixed", "l2block", "hot", "admm64", "hals_mu", "partitioned", "ablation"]
+    which = sys.argv[1:] or ["planted", "fixed", "l2block", "hot", "packed", "admm64", "hals_mu", "partitioned",
+                             "ablation"]
     if "planted" in which:
         p = datagen.planted_tiny(1)
         X = B.cstf_tensor_load_coo(p.dims, p.idx, p.vals)
@@ -63,6 +65,22 @@ def main():
         X.export_coo()
         del os.environ["CSTF_HOT_ROWS"]
         print("hot ok", flush=True)
+    if "packed" in which:
+        # packed 16-byte records forced on every 4-mode copy, hot-row flags in the keys,
+        # fast (R = 32) and generic (R = 5) kernels, export
+        os.environ["CSTF_PACK"] = "2"
+        os.environ["CSTF_HOT_ROWS"] = "100"
+        dims = (60, 2000, 700, 20)
+        idx, vals = datagen.coo(dims, (2, 2, 3, 1), 30000, 52)
+        X = B.cstf_tensor_load_coo(dims, idx, vals)
+        assert all(X.record_bytes(n) == 16 for n in range(4))
+        for R in (32, 5):
+            F = [cu(f) for f in datagen.init_factors(dims, R, 10)]
+            for n in range(4):
+                B.cstf_mttkrp(X, n, F, cu(np.zeros((dims[n], R))))
+        X.export_coo()
+        del os.environ["CSTF_PACK"], os.environ["CSTF_HOT_ROWS"]
+        print("packed ok", flush=True)
     if "admm64" in which:
         I, R = 20_003, 64          # 2,501 groups over <= 296 CTAs x 4 warps: several groups per warp
         rng = np.random.default_rng(1)

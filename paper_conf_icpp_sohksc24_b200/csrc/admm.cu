@@ -635,12 +635,22 @@ __global__ void __launch_bounds__(128) k_hals_rows(const double* __restrict__ M,
 #pragma unroll
     for (int k = 0; k < RP; k++) h[k] = th[lane * LD + k];
     for (int sw = 0; sw < sweeps; sw++) {
+      // S^T is loop-invariant: without this opaque copy of its address the compiler
+      // hoists all RP x RP shared loads out of the sweep loop and spills them (15 KB of
+      // local memory at RP = 32)
+      const double* STs = ST;
+      asm volatile("" : "+l"(STs));
 #pragma unroll
       for (int r = 0; r < RP; r++) {
-        const double d = ST[r * RP + r];
+        const double d = STs[r * RP + r];
+        const double2* Sr = reinterpret_cast<const double2*>(STs + r * RP);
         double dot = 0.0;
 #pragma unroll
-        for (int k = 0; k < RP; k++) dot = fma(h[k], ST[r * RP + k], dot);
+        for (int k = 0; k < RP; k += 2) {
+          const double2 sv = Sr[k / 2];
+          dot = fma(h[k], sv.x, dot);
+          dot = fma(h[k + 1], sv.y, dot);
+        }
         if (d > 0.0) {
           const double v = h[r] + (tm[lane * LD + r] - dot) / d;
           h[r] = v > 0.0 ? v : 0.0;

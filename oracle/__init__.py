@@ -21,7 +21,7 @@ _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
 OK, EINVAL, ENOMEM, NOT_SPD, NUMERIC = 0, 1, 3, 6, 7
-PROX_NONNEG, PROX_IDENTITY, PROX_L1, PROX_NONNEG_L1 = 0, 1, 2, 3
+PROX_NONNEG, PROX_IDENTITY, PROX_L1, PROX_NONNEG_L1, PROX_BOX = 0, 1, 2, 3, 4
 WARM_SCALED, WARM_NORMALIZED = 0, 1
 UPDATE_ADMM, UPDATE_HALS, UPDATE_MU = 0, 1, 2
 

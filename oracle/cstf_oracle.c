@@ -46,13 +46,17 @@
 #define PROX_IDENTITY 1 /* unconstrained (pin P10: reduces to CP-ALS, L360-368) */
 #define PROX_L1 2       /* r(H) = alpha ||H||_1: soft threshold at alpha/rho (L540-541, L615-619) */
 #define PROX_NONNEG_L1 3 /* r(H) = alpha ||H||_1 + indicator(R_+): max(0, x - alpha/rho) */
+#define PROX_BOX 4      /* indicator of the box [0, alpha] (alpha > 0): the projection min(max(x, 0), alpha)
+                           (reading D25; SURVEY f3 "box", L540-541 / L615-619: any element-wise operator) */
 
-/* Alg. 2 l.7: argmin_h r(h) + rho/2 (h - x)^2 for the element-wise regularisers above */
-static double prox_apply(int prox, double x, double tau) {
+/* Alg. 2 l.7: argmin_h r(h) + rho/2 (h - x)^2 for the element-wise regularisers above
+ * (tau = alpha / rho for the L1 thresholds; hi = alpha for the box) */
+static double prox_apply(int prox, double x, double tau, double hi) {
   switch (prox) {
     case PROX_IDENTITY: return x;
     case PROX_L1: return x > tau ? x - tau : (x < -tau ? x + tau : 0.0);
     case PROX_NONNEG_L1: return x > tau ? x - tau : 0.0;
+    case PROX_BOX: return x > 0.0 ? (x < hi ? x : hi) : 0.0;
     default: return x > 0.0 ? x : 0.0;
   }
 }
@@ -292,7 +296,8 @@ int oracle_cholesky(int R, const double* A, double* L) {
  *   H~ <- (L L^T)^{-1} (M + rho (H + U))      (l.6, row-major reading D1:
  *                                              forward then back substitution per row)
  *   H  <- prox(H~ - U)                        (l.7; nonneg: x > 0 ? x : +0.0, D15;
- *                                              L1 variants threshold at alpha/rho)
+ *                                              L1 variants threshold at alpha/rho,
+ *                                              the box clips to [0, alpha])
  *   U  <- U + H - H~                          (l.8)
  * until ||H - H~||^2 < eps ||H||^2 and ||H - H0||^2 < eps ||U||^2 (l.9, reading D3:
  *   squared norms of the UPDATED H, U, strict <, no division, at least one pass).
@@ -344,7 +349,7 @@ int oracle_admm(int64_t I, int R, const double* M, const double* S, double* H, d
         }
         for (int c = 0; c < R; c++) {
           double d = x[c] - u[c];
-          double hn = prox_apply(prox, d, tau);
+          double hn = prox_apply(prox, d, tau, alpha);
           double un = u[c] + hn - x[c];
           double e1 = hn - x[c], e2 = hn - h0[c];
           pr = pr + e1 * e1; ps = ps + e2 * e2; ph = ph + hn * hn; pu = pu + un * un;

@@ -24,7 +24,7 @@ c_void_p, c_int, c_int64, c_double = ctypes.c_void_p, ctypes.c_int, ctypes.c_int
 # status codes
 CSTF_OK, CSTF_ERR_INVALID_ARG, CSTF_ERR_UNSUPPORTED, CSTF_ERR_OUT_OF_MEMORY = 0, 1, 2, 3
 CSTF_ERR_CUDA, CSTF_ERR_NCCL, CSTF_ERR_NOT_SPD, CSTF_ERR_NUMERIC = 4, 5, 6, 7
-CSTF_PROX_NONNEG, CSTF_PROX_IDENTITY, CSTF_PROX_L1, CSTF_PROX_NONNEG_L1 = 0, 1, 2, 3
+CSTF_PROX_NONNEG, CSTF_PROX_IDENTITY, CSTF_PROX_L1, CSTF_PROX_NONNEG_L1, CSTF_PROX_BOX = 0, 1, 2, 3, 4
 CSTF_ADMM_AUTO, CSTF_ADMM_STREAMING, CSTF_ADMM_RESIDENT = 0, 1, 2
 CSTF_WARM_SCALED, CSTF_WARM_NORMALIZED = 0, 1
 CSTF_UPDATE_ADMM, CSTF_UPDATE_HALS, CSTF_UPDATE_MU = 0, 1, 2

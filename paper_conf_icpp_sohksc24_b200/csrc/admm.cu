@@ -61,11 +61,13 @@ struct KArgs {
 };
 
 // Alg. 2 l.7: argmin_h r(h) + rho/2 (h - x)^2 for the element-wise regularisers
-__device__ __forceinline__ double prox_apply(int prox, double x, double tau) {
+// (tau = alpha / rho for the L1 thresholds; hi = alpha for the box, reading D25)
+__device__ __forceinline__ double prox_apply(int prox, double x, double tau, double hi) {
   switch (prox) {
     case CSTF_PROX_IDENTITY: return x;
     case CSTF_PROX_L1: return x > tau ? x - tau : (x < -tau ? x + tau : 0.0);
     case CSTF_PROX_NONNEG_L1: return x > tau ? x - tau : 0.0;
+    case CSTF_PROX_BOX: return x > 0.0 ? (x < hi ? x : hi) : 0.0;
     default: return x > 0.0 ? x : 0.0;
   }
 }
@@ -323,7 +325,7 @@ __global__ void __launch_bounds__(kThreads, IREG ? 3 : 0) k_admm_dmma(KArgs a) {
           for (int i = 0; i < 2; i++) {
             const double ht = d[t][i];
             const double x = ht - u[t][i];
-            const double hn = prox_apply(a.prox, x, tau);
+            const double hn = prox_apply(a.prox, x, tau, a.alpha);
             const double un = hn - x;         // U + H - H~ with x = H~ - U (one op)
             const double e1 = hn - ht, e2 = hn - h[t][i];
             pr = fma(e1, e1, pr); ps = fma(e2, e2, ps); ph = fma(hn, hn, ph); pu = fma(un, un, pu);
@@ -339,7 +341,7 @@ __global__ void __launch_bounds__(kThreads, IREG ? 3 : 0) k_admm_dmma(KArgs a) {
           for (int i = 0; i < 2; i++) {
             const double ht = d[t][i];
             const double x = ht - u[t][i];
-            const double hn = prox_apply(a.prox, x, tau);
+            const double hn = prox_apply(a.prox, x, tau, a.alpha);
             u[t][i] = hn - x;
             h[t][i] = hn;
           }
@@ -537,7 +539,7 @@ __global__ void __launch_bounds__(128) k_admm_generic(KArgs a) {
         for (int k = 0; k < R; k++) ht = fma(st[k], sinv[k * R + tid], ht);
       __syncthreads();
       const double x = ht - u;
-      const double hn = prox_apply(a.prox, x, tau);
+      const double hn = prox_apply(a.prox, x, tau, a.alpha);
       const double un = (u + hn) - ht;
       const double e1 = hn - ht, e2 = hn - h;
       if (cok) {

@@ -262,7 +262,8 @@ cstf_status factorize_impl(const cstf_tensor* X, const cstf_opts* o, const cstf_
   auto setup = [&]() -> cstf_status {
     if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
     if (o->outer_iters < 1 || o->admm.max_iter < 1) return fail(CSTF_ERR_INVALID_ARG, "outer_iters/max_iter < 1");
-    if (o->admm.prox < CSTF_PROX_NONNEG || o->admm.prox > CSTF_PROX_NONNEG_L1 || !(o->admm.alpha >= 0.0))
+    if (o->admm.prox < CSTF_PROX_NONNEG || o->admm.prox > CSTF_PROX_BOX || !(o->admm.alpha >= 0.0) ||
+        (o->admm.prox == CSTF_PROX_BOX && !(o->admm.alpha > 0.0)))
       return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
     if (o->update < CSTF_UPDATE_ADMM || o->update > CSTF_UPDATE_MU) return fail(CSTF_ERR_INVALID_ARG, "unknown update");
     if (o->update == CSTF_UPDATE_MU && R > 64) return fail(CSTF_ERR_UNSUPPORTED, "MU update for R > 64");
@@ -647,7 +648,8 @@ cstf_status cstf_admm_update(const double* d_M, const double* d_S, double* d_H, 
     return fail(CSTF_ERR_INVALID_ARG, "NULL argument or I < 0");
   if (!rank_ok(R)) return fail(CSTF_ERR_UNSUPPORTED, "R must be in [1, 128]");
   if (opts->max_iter < 1 || opts->tol < 0.0) return fail(CSTF_ERR_INVALID_ARG, "max_iter < 1 or tol < 0");
-  if (opts->prox < CSTF_PROX_NONNEG || opts->prox > CSTF_PROX_NONNEG_L1 || !(opts->alpha >= 0.0))
+  if (opts->prox < CSTF_PROX_NONNEG || opts->prox > CSTF_PROX_BOX || !(opts->alpha >= 0.0) ||
+      (opts->prox == CSTF_PROX_BOX && !(opts->alpha > 0.0)))
     return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
   cudaStream_t st = S(stream);
   DriverWs& w = dws();

@@ -484,6 +484,49 @@ def test_factorize_nonneg_l1(B):
     assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
 
 
+@pytest.mark.parametrize("tol", [0.0, 1e-2])
+@pytest.mark.parametrize("R,variant", [(8, 0), (32, 0), (32, 1), (64, 0), (100, 0)])
+def test_admm_box_prox(B, R, variant, tol):
+    """f3 (reading D25): the indicator of the box [0, alpha] in the fused kernel vs the
+    oracle; alpha below the largest unconstrained value, so both bounds are active."""
+    M, S, H, U = admm_inputs(1500, R, 11 + R)
+    Hn, _, _ = oracle.admm(M, S, H, U, tol=0.0, max_iter=10)
+    alpha = 0.5 * float(np.max(Hn))
+    Hd, Ud = cu(H), cu(U)
+    st = B.cstf_admm_update(cu(M), cu(S), Hd, Ud, tol=tol, max_iter=10, prox=B.CSTF_PROX_BOX, alpha=alpha,
+                            variant=variant)
+    Hr, Ur, sr = oracle.admm(M, S, H, U, tol=tol, max_iter=10, prox=oracle.PROX_BOX, alpha=alpha)
+    assert st["iters"] == sr["iters"]
+    assert normwise(host(Hd), Hr) <= TOL and normwise(host(Ud), Ur) <= TOL
+    got = host(Hd)
+    assert np.any(got == 0.0) and np.any(got == alpha) and got.max() <= alpha
+
+
+def test_box_prox_rejects_nonpositive_bound(B):
+    M, S, H, U = admm_inputs(100, 8, 3)
+    with pytest.raises(B.CstfError):
+        B.cstf_admm_update(cu(M), cu(S), cu(H), cu(U), prox=B.CSTF_PROX_BOX, alpha=0.0)
+
+
+def test_factorize_box(B):
+    """factorize with the box prox (alpha = 5, active: the oracle's fit differs from the
+    plain non-negative run) against the oracle: counts, fits, factors."""
+    c = datagen.CONFIGS["nell2"].scaled(40, nnz_factor=800)
+    idx, vals = c.generate()
+    start = datagen.init_factors(c.dims, 16, c.seed)
+    ref = oracle.coalesce(c.dims, idx, vals)
+    orc = oracle.factorize(ref, start, outer_iters=5, tol=1e-2, max_iter=10, prox=oracle.PROX_BOX, alpha=5.0)
+    X = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    F = [cu(f) for f in start]
+    lam = cu(np.zeros(16))
+    gpu = B.cstf_factorize(X, F, lam, B.make_opts(16, outer_iters=5, tol=1e-2, prox=B.CSTF_PROX_BOX, alpha=5.0))
+    n, tie = compare_iteration_counts(gpu["iters"], orc, 1e-2)
+    assert tie is None
+    assert np.max(np.abs(gpu["fit"] - orc["fit"]) / np.abs(orc["fit"])) <= 1e-6
+    for a, b in zip(F, orc["factors"]):
+        assert normwise(host(a), b) <= 1e-6
+
+
 @pytest.mark.parametrize("update", ["hals", "mu"])
 @pytest.mark.parametrize("I,R", [(1, 8), (1003, 8), (3001, 32), (999, 64), (300, 100)])
 def test_hals_mu_updates(B, update, I, R):

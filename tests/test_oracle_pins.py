@@ -446,6 +446,53 @@ def test_f3_l1_with_zero_alpha_is_the_plain_operator(rng):
     assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
 
 
+def box_bruteforce(S, m, hi):
+    """min_h 1/2 h^T S h - m^T h over the box 0 <= h <= hi (S SPD), by enumerating for
+    every coordinate the state lower bound / free / upper bound (3^R patterns) and
+    keeping the feasible stationary point of least objective."""
+    from itertools import product
+    R = len(m)
+    best, best_h = np.inf, None
+    for pat in product((0, 1, 2), repeat=R):
+        h = np.where(np.array(pat) == 2, hi, 0.0)
+        F = [i for i in range(R) if pat[i] == 1]
+        if F:
+            C = [i for i in range(R) if pat[i] != 1]
+            rhs = m[F] - (S[np.ix_(F, C)] @ h[C] if C else 0.0)
+            h[F] = np.linalg.solve(S[np.ix_(F, F)], rhs)
+            if np.any(h[F] < 0.0) or np.any(h[F] > hi):
+                continue
+        f = 0.5 * h @ S @ h - m @ h
+        if f < best:
+            best, best_h = f, h
+    return best_h
+
+
+@pytest.mark.parametrize("R", [2, 3])
+def test_f3_box_fixed_point_is_bruteforce_qp(rng, R):
+    """Reading D25: ADMM with the indicator of [0, alpha] converges to the box-constrained
+    least-squares minimiser found by brute force; both bounds are active somewhere."""
+    S = make_S(rng, R)
+    I = 40
+    M = (rng.random((I, R)) - 0.3) * 2.0 * np.diag(S).mean()
+    hi = 0.6
+    H, U, st = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), tol=0.0, max_iter=6000,
+                           prox=oracle.PROX_BOX, alpha=hi)
+    ref = np.array([box_bruteforce(S, M[i], hi) for i in range(I)])
+    assert np.any(ref == 0.0) and np.any(ref == hi)
+    assert normwise(H, ref) <= 1e-9
+
+
+def test_f3_box_with_unreachable_bound_is_the_plain_operator(rng):
+    """A box whose upper bound is never reached runs exactly the non-negativity operator."""
+    R, I = 5, 40
+    S = make_S(rng, R)
+    M = rng.random((I, R)) - 0.5
+    a = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), max_iter=20, prox=oracle.PROX_BOX, alpha=1e300)
+    b = oracle.admm(M, S, np.zeros((I, R)), np.zeros((I, R)), max_iter=20, prox=oracle.PROX_NONNEG)
+    assert np.array_equal(a[0], b[0]) and np.array_equal(a[1], b[1])
+
+
 # --------------------------------------------------------------------- f1: HALS / MU
 def nnls_objective(S, M, H):
     return float(np.sum(0.5 * np.einsum("ir,rs,is->i", H, S, H) - np.einsum("ir,ir->i", M, H)))

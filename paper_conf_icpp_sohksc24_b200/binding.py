@@ -177,9 +177,9 @@ class Comm:
         _check(_lib.cstf_comm_info(self.handle, ctypes.byref(n), ctypes.byref(r)), "cstf_comm_info")
         return n.value, r.value
 
-    def __del__(self):
+    def __del__(self, _destroy=_lib.cstf_comm_destroy):
         if getattr(self, "handle", None):
-            _lib.cstf_comm_destroy(self.handle)
+            _destroy(self.handle)
             self.handle = None
 
 
@@ -293,9 +293,10 @@ class Tensor:
                                            vals.ctypes.data), "cstf_tensor_export_coo")
         return idx, vals
 
-    def free(self):
-        if self.handle:
-            _lib.cstf_tensor_free(self.handle)
+    def free(self, _free=_lib.cstf_tensor_free):
+        # _free bound at definition: at interpreter exit the module global may be gone
+        if getattr(self, "handle", None):
+            _free(self.handle)
             self.handle = None
 
     def __del__(self):

@@ -119,9 +119,11 @@ struct ModeStore {
   // Packed 16-byte records (round 2): when the row indices of
   // the N-1 = 3 gathered slots fit one 64-bit word, record = {uint64 key, f64 x} with
   // slot q at bits [pk_sh[q], pk_sh[q] + width) of key: the row, or pk_hot[q] | hot slot
-  // (pk_hot[q] = the field's top bit, 0 for slots without hot rows).  Not for L2-blocked
-  // copies.  CSTF_PACK=0 keeps the 32-byte records.
+  // (pk_hot[q] = the field's top bit, 0 for slots without hot rows).  In an L2-blocked
+  // copy the blocked slot stores its row within the block (pk_rel = tslot; the block is
+  // the one of the virtual row).  CSTF_PACK=0 keeps the 32-byte records.
   bool pk = false;
+  int pk_rel = -1;          // L2-blocked packed copy: slot tslot holds the row within its block
   int pk_sh[7] = {0};
   uint32_t pk_mask[7] = {0};
   uint32_t pk_hot[7] = {0};

@@ -81,6 +81,9 @@ struct MArgs {
   const double* HF[7];  // hot-row table of the factor of slot q (records 0x80000000 | hot slot), or null
   int l2blocked;        // launch over an L2-blocked copy (rows are virtual rows)
   int pk;               // packed 16-byte records (ModeStore::pk): slot q = (key >> pk_sh[q]) & pk_mask[q]
+  int pk_rel;           // L2-blocked packed copy: slot stored relative to its block (-1: none)
+  uint32_t pk_blk;      //   rows per block of that slot
+  int64_t Iout;         //   output rows per block (virtual row v lies in block v / Iout)
   int pk_sh[3];
   uint32_t pk_mask[3], pk_hot[3];
 };
@@ -164,7 +167,7 @@ __device__ __forceinline__ const double2* row_addr(const char* base, unsigned j)
 // One warp processes chunk c.  Fb[q] = lane's byte offset into the row source of
 // slot q (a factor in global memory, or the shared-memory slab of a k-blocked
 // copy, already shifted by the slab's first row).
-template <int NOTHER, int R, int RECB, int GL = 0, bool HOT = false, int UNR = 1>
+template <int NOTHER, int R, int RECB, int GL = 0, bool HOT = false, int UNR = 1, bool REL = false>
 __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const char* const* Fb, int4* srec,
                                               const char* const* HFb = nullptr) {
   constexpr int RV = R / 2;                    // double2 per row
@@ -186,6 +189,15 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
 #pragma unroll
     for (int s = 0; s < VPL; s++) acc[s] = make_double2(0.0, 0.0);
     int64_t seg_end = (row < row_end) ? min(a.rowptr[row + 1], p1) : p1;
+    // REL (packed L2-blocked copy): the blocked slot's field is the row within the block of
+    // the current virtual row; kbrow = that block's first row, advanced at block changes
+    uint32_t kbrow = 0;
+    int64_t kb_next = 0;
+    if constexpr (REL) {
+      const int64_t kb = row / a.Iout;
+      kbrow = (uint32_t)kb * a.pk_blk;
+      kb_next = (kb + 1) * a.Iout;
+    }
 
     auto flush = [&](int64_t r) {
 #pragma unroll
@@ -231,6 +243,9 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
           flush(row);
           row++;
           seg_end = min(a.rowptr[row + 1], p1);
+          if constexpr (REL) {
+            if (row >= kb_next) { kbrow += a.pk_blk; kb_next += a.Iout; }
+          }
           continue;
         }
         const int run = (int)min((int64_t)(nb - t), seg_end - p);
@@ -257,6 +272,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
                 const char* base;
                 unsigned j;
                 slot_row<PK, HOT>(a, qq, w, Fb[qq], HOT ? HFb[qq] : nullptr, base, j);
+                if constexpr (REL) j += (qq == a.pk_rel) ? kbrow : 0u;
                 const double2* rp = row_addr<ROWB>(base, j);
 #pragma unroll
                 for (int s = 0; s < VPL; s++) xs[u][qq][s] = rp[s * G];
@@ -293,6 +309,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
             const char* base;
             unsigned j;
             slot_row<PK, HOT>(a, qq, w, Fb[qq], HOT ? HFb[qq] : nullptr, base, j);
+                if constexpr (REL) j += (qq == a.pk_rel) ? kbrow : 0u;
             const double2* rp = row_addr<ROWB>(base, j);
 #pragma unroll
             for (int s = 0; s < VPL; s++) {
@@ -318,7 +335,7 @@ __device__ __forceinline__ void process_chunk(const MArgs& a, int64_t c, const c
 }
 
 // MINB: CTAs per SM the register budget targets (2 for long rows, 4 for short ones)
-template <int NOTHER, int R, int RECB, int MINB, int GL = 0, bool HOT = false, int UNR = 1>
+template <int NOTHER, int R, int RECB, int MINB, int GL = 0, bool HOT = false, int UNR = 1, bool REL = false>
 __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
   constexpr int G = GL ? GL : ((R / 2) < 32 ? (R / 2) : 32);
   const int gl = (threadIdx.x & 31) % G;
@@ -343,11 +360,11 @@ __global__ void __launch_bounds__(kWarps * 32, MINB) k_mttkrp_fast(MArgs a) {
       if ((threadIdx.x & 31) == 0) c = atomicAdd(a.queue, 1ULL);
       c = __shfl_sync(0xffffffffu, c, 0);
       if ((int64_t)c >= a.nchunks) break;
-      process_chunk<NOTHER, R, RECB, GL, HOT, UNR>(a, (int64_t)c, Fb, srec, HFb);
+      process_chunk<NOTHER, R, RECB, GL, HOT, UNR, REL>(a, (int64_t)c, Fb, srec, HFb);
     }
     return;
   }
-  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT, UNR>(a, c, Fb, srec, HFb);
+  for (int64_t c = warp0; c < a.nchunks; c += nwarps) process_chunk<NOTHER, R, RECB, GL, HOT, UNR, REL>(a, c, Fb, srec, HFb);
 }
 
 // k-blocked copy: CTA chunk b (8 warp chunks) lies in block kb = ckb[b]; the
@@ -394,6 +411,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
     int64_t seg0 = max(a.rowptr[row < row_end ? row : 0], p0);
     for (; row < row_end; row++) {
       const int64_t seg1 = min(a.rowptr[row + 1], p1);
+      const unsigned kbrow = a.pk_rel >= 0 ? (unsigned)(row / a.Iout) * a.pk_blk : 0u;   // block-relative slot
       double acc[CPL];
 #pragma unroll
       for (int s = 0; s < CPL; s++) acc[s] = 0.0;
@@ -408,6 +426,7 @@ __global__ void __launch_bounds__(kWarps * 32) k_mttkrp_generic(MArgs a) {
             const unsigned f = pk_field(a, q, reinterpret_cast<const unsigned*>(r)[0], reinterpret_cast<const unsigned*>(r)[1]);
             j = f & ~a.pk_hot[q];
             if (f & a.pk_hot[q]) fq = a.HF[q];
+            else if (q == a.pk_rel) j += kbrow;
           } else if ((int)j < 0) {
             fq = a.HF[q];                   // hot row (hot-row table)
             j &= 0x7fffffffu;
@@ -530,6 +549,19 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
   const int minb = mttkrp_minb(a.nnz, a.I - a.rbase, a.R, a.l2blocked != 0, hot, NOTHER);
   const bool short_rows = minb == 4;
   const bool mid_rows = minb == 3;
+  if constexpr (RECB == 16 && NOTHER == 3) {
+    if (a.pk_rel >= 0) {   // packed L2-blocked copy (block-relative slot): R = 32 / 64 kernels, else generic
+#define RCASE(RR, GG, HH)                                                                                    \
+  if (a.R == RR && gl == GG && hot == HH) {                                                                \
+    if (short_rows) k_mttkrp_fast<NOTHER, RR, RECB, 4, GG, HH, 1, true><<<grid, kWarps * 32, 0, st>>>(a);     \
+    else k_mttkrp_fast<NOTHER, RR, RECB, 2, GG, HH, 1, true><<<grid, kWarps * 32, 0, st>>>(a);                \
+    return true;                                                                                           \
+  }
+      RCASE(32, 0, false) RCASE(32, 0, true) RCASE(32, 8, false) RCASE(64, 0, false) RCASE(64, 0, true)
+#undef RCASE
+      return false;
+    }
+  }
   if (tiled) {
     switch (a.R) {     // slab = 256 rows x R doubles: 2 KB .. 128 KB
       case 8: return launch_tiled_r<NOTHER, RECB, 8>(a, grid, st);
@@ -919,6 +951,9 @@ cstf_status mttkrp(const cstf_tensor* X, int mode, int R, const double* const* d
   a.recb = ms.recb;
   a.pk = ms.pk ? 1 : 0;
   for (int q = 0; q < 3; q++) { a.pk_sh[q] = ms.pk_sh[q]; a.pk_mask[q] = ms.pk_mask[q]; a.pk_hot[q] = ms.pk_hot[q]; }
+  a.pk_rel = ms.pk_rel;
+  a.pk_blk = ms.pk_rel >= 0 ? (uint32_t)ms.blk_rows : 1u;
+  a.Iout = ms.I > 0 ? ms.I : 1;
   a.nother = N - 1;
   for (int q = 0; q < N - 1; q++) a.F[q] = d_factors[ms.other[q]];
   a.It = X->dims[ms.other[N - 2]];      // slab blocks: rows of the last slot's factor

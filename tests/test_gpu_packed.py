@@ -2,8 +2,9 @@
 decide_pack, mttkrp.cu pk_field): {uint64 bit-packed indices of the three gathered
 modes (plus hot-row flags), f64 value} instead of {3 x int32, pad, f64}.
 
-  * chosen where the three fields fit 64 bits, the copy is not L2-blocked and has
-    >= 16 nonzeros per row (CSTF_PACK=2 forces it wherever the fields fit);
+  * chosen where the three fields fit 64 bits (an L2-blocked copy stores its blocked
+    slot relative to the block) and the copy has >= 16 nonzeros per (virtual) row
+    (CSTF_PACK=2 forces it wherever the fields fit);
   * MTTKRP on packed copies equals the 32-byte-record copies bit for bit (same nonzero
     order, same kernels and arithmetic) for the fast kernel (R = 16 / 32 / 64, with and
     without hot-row slots, both group widths) and the generic kernel (R = 5), and the
@@ -94,8 +95,10 @@ def test_packed_mttkrp_bitwise_and_oracle(B, delicious_small, hot, R, g, monkeyp
 def test_packed_only_where_fields_fit(B, monkeypatch):
     """Mode 0 of a tensor whose three other modes need 22 bits each (66 > 64) keeps the
     32-byte records; the other modes (one 2-bit field) pack (forced past the row-length
-    rule).  MTTKRP of both kinds against the oracle."""
+    rule; L2 blocks off, which would make mode 0's longest slot block-relative and fit).
+    MTTKRP of both kinds against the oracle."""
     monkeypatch.setenv("CSTF_PACK", "2")
+    monkeypatch.setenv("CSTF_L2_BLOCK", "0")
     dims = (3, 3_000_000, 2_500_000, 2_200_000)
     need = [sum(bits(dims[k]) for k in range(4) if k != n) for n in range(4)]
     assert need[0] > 64 and all(x <= 64 for x in need[1:])
@@ -110,21 +113,36 @@ def test_packed_only_where_fields_fit(B, monkeypatch):
         assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, n
 
 
-def test_l2_blocked_copies_not_packed(B, delicious_small, monkeypatch):
-    """L2-blocked copies (forced) keep 32-byte records; unblocked ones of the same store pack."""
+@pytest.mark.parametrize("hot", [None, "300"])
+@pytest.mark.parametrize("R", [32, 64, 5])
+def test_l2_blocked_copies_pack_block_relative(B, delicious_small, hot, R, monkeypatch):
+    """L2-blocked copies (forced 20,000-row blocks) pack too, their blocked slot stored as
+    the row within its block (the kernel adds the block's first row of the current virtual
+    row): MTTKRP bit for bit equal to the 32-byte copies and to the oracle within 1e-9,
+    export (mode 0 is blocked here) back to the canonical tensor."""
     c, idx, vals, ref = delicious_small
     monkeypatch.setenv("CSTF_PACK", "2")
     monkeypatch.setenv("CSTF_L2_BLOCK_ROWS", "20000")
+    if hot:
+        monkeypatch.setenv("CSTF_HOT_ROWS", hot)
     X = B.cstf_tensor_load_coo(c.dims, idx, vals)
-    kinds = [(X.layout(n)[0] > 1, X.record_bytes(n)) for n in range(4)]
-    assert any(blk for blk, _ in kinds)
-    for blk, rb in kinds:
-        assert rb == (32 if blk else 16)
-    R = 32
+    monkeypatch.setenv("CSTF_PACK", "0")
+    Xu = B.cstf_tensor_load_coo(c.dims, idx, vals)
+    blocked = [X.layout(n)[0] > 1 for n in range(4)]
+    assert blocked[0] and sum(blocked) >= 2
+    assert [X.record_bytes(n) for n in range(4)] == [16] * 4
+    assert [Xu.record_bytes(n) for n in range(4)] == [32] * 4
     F = datagen.init_factors(c.dims, R, 23)
     Fd = [cu(f) for f in F]
-    for n, got in enumerate(mttkrp_all(B, X, c.dims, Fd, R)):
-        assert normwise(got, oracle.mttkrp(ref, n, F)) <= TOL, n
+    a = mttkrp_all(B, X, c.dims, Fd, R)
+    b = mttkrp_all(B, Xu, c.dims, Fd, R)
+    for n in range(4):
+        assert np.array_equal(a[n], b[n]), n
+        assert normwise(a[n], oracle.mttkrp(ref, n, F)) <= TOL, n
+    gi, gv = X.export_coo()
+    for m in range(4):
+        assert np.array_equal(gi[m], ref.idx[m]), m
+    assert np.array_equal(gv, ref.vals)
 
 
 def test_packed_export_with_hot_rows(B, delicious_small, monkeypatch):

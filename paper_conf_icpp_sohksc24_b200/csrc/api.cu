@@ -650,7 +650,7 @@ cstf_status cstf_admm_update(const double* d_M, const double* d_S, double* d_H, 
   if (opts->max_iter < 1 || opts->tol < 0.0) return fail(CSTF_ERR_INVALID_ARG, "max_iter < 1 or tol < 0");
   if (opts->prox < CSTF_PROX_NONNEG || opts->prox > CSTF_PROX_BOX || !(opts->alpha >= 0.0) ||
       (opts->prox == CSTF_PROX_BOX && !(opts->alpha > 0.0)))
-    return fail(CSTF_ERR_INVALID_ARG, "unknown prox or alpha < 0");
+    return fail(CSTF_ERR_INVALID_ARG, "unknown prox, alpha < 0, or box bound alpha <= 0");
   cudaStream_t st = S(stream);
   DriverWs& w = dws();
   CSTF_TRY(w.inv.ensure((size_t)R * R * 8));

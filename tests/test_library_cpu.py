@@ -65,6 +65,15 @@ def test_argument_validation_without_gpu(lib):
     assert st == lib.CSTF_ERR_INVALID_ARG
     st = lib._lib.cstf_gram(ctypes.c_void_p(8), 4, 129, ctypes.c_void_p(8), None, None)
     assert st == lib.CSTF_ERR_UNSUPPORTED
+    # the box prox needs a positive upper bound (reading D25); checked before any device work
+    d = ctypes.c_void_p(8)
+    o = lib.admm_opts(max_iter=10, prox=lib.CSTF_PROX_BOX, alpha=0.0)
+    st = lib._lib.cstf_admm_update(d, d, d, d, 16, 8, ctypes.byref(o), None, None, None)
+    assert st == lib.CSTF_ERR_INVALID_ARG and b"box" in lib._lib.cstf_last_error_message()
+    o = lib.admm_opts(max_iter=10, prox=5)
+    assert lib._lib.cstf_admm_update(d, d, d, d, 16, 8, ctypes.byref(o), None, None, None) == lib.CSTF_ERR_INVALID_ARG
+    rb = ctypes.c_int()
+    assert lib._lib.cstf_tensor_record_bytes(None, 0, ctypes.byref(rb)) == lib.CSTF_ERR_INVALID_ARG
 
 
 def check_partition(counts, P, owner, local):

@@ -445,7 +445,8 @@ def main():
             "roofline": roof, "roofline_admm": roof_admm, "admm_update_gbs": admm_gbs,
             "phases_ms_per_step": phase_ms, "clocks": clk,
             "setup": {"generate_s": t_gen, "load_coo_s": t_load, "nnz_coalesced": nnz,
-                      "layout": [dict(zip(("nblk", "blk_rows", "blk_mode"), X.layout(n))) for n in range(N)]}}
+                      "layout": [dict(zip(("nblk", "blk_rows", "blk_mode"), X.layout(n)),
+                                      record_bytes=X.record_bytes(n)) for n in range(N)]}}
     # end to end through the public API with HOST buffers (pinned), one outer iteration per step
     if not args.no_e2e:
         hf = [torch.from_numpy(f.copy()).pin_memory() for f in F0]

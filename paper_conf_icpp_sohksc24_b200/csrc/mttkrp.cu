@@ -50,6 +50,17 @@ int mttkrp_minb(int64_t nnz, int64_t rows, int R, bool tiled, bool hot = false, 
   return 2;
 }
 
+// Hot-row copies of 4-mode tensors at R = 32 with >= 16 nonzeros per row (not L2-blocked):
+// 8-lane groups with 2 steps of row loads in flight (Delicious mode 0 9.19 -> 8.99 ms,
+// mode 2 9.36 -> 9.12 ms; short rows stay on 16-lane groups: mode 1 11.26 -> 11.56 ms with
+// 8; profiles/r02_mttkrp_g8_hot_probe.txt).  The group width depends on the row class only,
+// so forced unroll depths (CSTF_MTTKRP_UNR) keep the accumulation order.
+bool mttkrp_hot_g8(int64_t nnz, int64_t rows, int R, bool tiled, bool hot, int nother) {
+  if (!(hot && R == 32 && !tiled && nother == 3 && nnz >= 16 * rows)) return false;
+  const char* ge = getenv("CSTF_MTTKRP_G");      // CSTF_MTTKRP_G=0: 16-lane groups everywhere (tests)
+  return !(ge && atoi(ge) == 0);
+}
+
 // Steps of row gathers issued before the first product (hot-row copies, R = 32; 1 elsewhere)
 int mttkrp_unr(int64_t nnz, int64_t rows, int R, bool tiled, bool hot, int nother = 3) {
   if (!hot || R != 32 || nother > 4) return 1;
@@ -57,6 +68,7 @@ int mttkrp_unr(int64_t nnz, int64_t rows, int R, bool tiled, bool hot, int nothe
     const int v = atoi(e);
     if (v >= 1 && v <= 4) return v;
   }
+  if (mttkrp_hot_g8(nnz, rows, R, tiled, hot, nother)) return 2;
   if (tiled || nnz >= 64 * rows) return 1;
   return nnz < 16 * rows ? 2 : 4;
 }
@@ -590,6 +602,19 @@ bool launch_fast(const MArgs& a, int grid, cudaStream_t st, bool tiled, int gl, 
     else k_mttkrp_fast<NOTHER, 32, RECB, 2, 0, true, UU><<<grid, kWarps * 32, 0, st>>>(a);              \
     return true;                                                                                       \
   }
+    // medium and long rows of hot-row copies (4-mode, R = 32, >= 16 nonzeros per row): 8-lane
+    // groups, 4 nonzeros per warp step (mttkrp_hot_g8)
+    if constexpr (NOTHER == 3) {
+      if (mttkrp_hot_g8(a.nnz, a.I - a.rbase, a.R, a.l2blocked != 0, hot, NOTHER)) {
+#define G8CASE(UU)                                                                                        \
+  if (unr == UU) {                                                                                        \
+    k_mttkrp_fast<NOTHER, 32, RECB, 2, 8, true, UU><<<grid, kWarps * 32, 0, st>>>(a);                       \
+    return true;                                                                                          \
+  }
+        G8CASE(1) G8CASE(2) G8CASE(3) G8CASE(4)
+#undef G8CASE
+      }
+    }
     UCASE(2) UCASE(3) UCASE(4)
 #undef UCASE
   }
